@@ -1,0 +1,213 @@
+"""Pins for the CPU oracle (oracle/), each against something other than the oracle itself:
+values the paper prints, closed forms, textbook identities, brute force on tiny inputs,
+and digests from an independent implementation (tests/golden/)."""
+import hashlib
+import json
+import os
+
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _bits(words, pos, b):
+    """read b bits at stream position pos, LSB-first (test-side reader)."""
+    v = 0
+    for k in range(b):
+        bit = pos + k
+        v |= ((int(words[bit // 32]) >> (bit % 32)) & 1) << k
+    return v
+
+
+# ---------------------------------------------------------------- FOR layout
+def test_fig4_worked_example():
+    """P:679-698 Figure 4: reference 99, bitwidths 2 and 4, codes of P:681."""
+    g = json.load(open(os.path.join(GOLD, "fig4.json")))
+    e = oracle.for_encode(np.array(g["values"], np.int32), block_size=16, mb_count=2)
+    d = e["data"]
+    assert list(e["header"]) == [16, 2, 16]
+    assert list(e["starts"]) == [0, 4]
+    assert int(d[0]) == g["reference"] == 99
+    assert [int(d[1]) & 255, (int(d[1]) >> 8) & 255] == g["bitwidths"]
+    # codes of the value row, read back from the packed miniblocks
+    codes = [_bits(d[2:3], 2 * i, 2) for i in range(8)] + [_bits(d[3:4], 4 * i, 4) for i in range(8)]
+    assert codes == g["codes"]
+    assert [int(w) for w in d] == g["words"]
+    assert list(oracle.for_decode(e)) == g["values"]
+
+
+def test_range_100_130_needs_5_bits():
+    """values in [100,130], reference 100, log2(130+1-100) -> 5 bits."""
+    x = np.array([100 + (i * 7) % 31 for i in range(127)] + [130], np.int32)
+    assert x.min() == 100 and x.max() == 130
+    e = oracle.for_encode(x)
+    assert int(e["data"][0]) == 100
+    bw = int(e["data"][1])
+    assert max((bw >> (8 * j)) & 255 for j in range(4)) == 5
+
+
+def test_algorithm1_block_sizes():
+    """Alg. 1 lines 7-14: a miniblock at b bits occupies b words, after a
+    2-word header, so block i spans 2 + sum_j b_ij words."""
+    rng = np.random.default_rng(5)
+    x = np.concatenate([rng.integers(0, 2**b, 128, dtype=np.int32) for b in (0, 3, 17, 31, 1)])
+    e = oracle.for_encode(x)
+    s, d = e["starts"], e["data"]
+    for i in range(len(s) - 1):
+        bw = int(d[s[i] + 1])
+        assert s[i + 1] - s[i] == 2 + sum((bw >> (8 * j)) & 255 for j in range(4))
+
+
+def test_for_overhead_uniform():
+    """GPU-FOR overhead = 0.75 bit/int on uniform [0, 2^b)."""
+    n = 512 * 200
+    for b in (1, 4, 8, 16, 24, 31):
+        x = datagen.uniform_bits(b, n, seed=11 + b)
+        bits = 8 * oracle.for_encode(x).nbytes() / n
+        nb = n // 128
+        assert oracle.for_encode(x).nbytes() == 4 * (3 + nb + 1 + nb * (2 + 4 * b))
+        assert abs(bits - (b + 0.75)) < 2e-3  # header + final start word: 128 bits / n
+
+
+def test_dfor_overhead_uniform():
+    """GPU-DFOR = 0.81 bit/int overhead (+1 first value per D=4 blocks)
+    plus one extra bit because deltas of random data span twice the range."""
+    n = 512 * 200
+    for b in (2, 8, 16, 30):
+        x = datagen.uniform_bits(b, n, seed=21 + b)
+        bits = 8 * oracle.dfor_encode(x).nbytes() / n
+        assert abs(bits - (b + 1 + 0.8125)) < 2e-3
+
+
+def test_sorted_d1_sizes_match_paper():
+    """P:1701-1705 (and P:1075-1079): D1 with 2^28 unique values over 250M entries:
+    GPU-DFOR 1.8 and GPU-FOR 7.8 bits per int.  The column is evenly spread, so its
+    first 1M entries have the same per-tile structure."""
+    x = datagen.d1_prefix(1_000_000, 2**28, 250_000_000)
+    f = 8 * oracle.for_encode(x).nbytes() / len(x)
+    d = 8 * oracle.dfor_encode(x).nbytes() / len(x)
+    assert round(f, 1) == 7.8 and round(d, 1) == 1.8
+    assert abs(f - 7.75) < 1e-3 and abs(d - 1.8125) < 2e-3
+
+
+# ---------------------------------------------------------------- RLE example
+def test_rle_example():
+    """(x,x,x,x,y,y,z,z,z) -> values (x,y,z), run lengths (4,2,3)."""
+    xx, yy, zz = 7, -3, 1000
+    col = np.array([xx] * 4 + [yy] * 2 + [zz] * 3, np.int32)
+    e = oracle.rfor_encode(col)
+    dV, dL = e["dataV"], e["dataL"]
+    assert int(dV[0]) == 3 and int(dL[0]) == 3          # run / value count word
+    refV, refL = np.int32(dV[1]), np.int32(dL[1])
+    bV, bL = int(dV[2]) & 255, int(dL[2]) & 255
+    V = [int(refV) + _bits(dV[6:], bV * i, bV) for i in range(3)]
+    L = [int(refL) + _bits(dL[6:], bL * i, bL) for i in range(3)]
+    assert V == [xx, yy, zz] and L == [4, 2, 3]
+    assert list(oracle.rfor_decode(e)) == list(col)
+
+
+# ---------------------------------------------------------------- brute force
+def test_bruteforce_all_tiny_columns_roundtrip():
+    """Every column of length <= 4 over {INT32_MIN,-1,0,1,2,3,INT32_MAX} (2,801 columns)."""
+    count = 0
+    for x in datagen.small_alphabet_columns(4):
+        for s in ("for", "dfor", "rfor"):
+            e = oracle.encode(s, x)
+            assert np.array_equal(oracle.decode(e), x), (s, x)
+        count += 1
+    assert count == 2801
+
+
+def test_mixed_ragged_roundtrip():
+    for name, x in datagen.mixed_columns():
+        for s in ("for", "dfor", "rfor"):
+            e = oracle.encode(s, x)
+            assert np.array_equal(oracle.decode(e), x), (s, name)
+
+
+def test_dfor_is_first_plus_exclusive_cumsum():
+    """delta decode == prefix sum; textbook check with np.cumsum per tile."""
+    x = datagen.near_sorted(512 * 9 + 77, seed=3)
+    e = oracle.dfor_encode(x)
+    s, d = e["starts"], e["data"]
+    # first values sit one word before the tile's first block (Fig. 6)
+    firsts = [np.int32(d[s[4 * t] - 1]) for t in range((len(x) + 511) // 512)]
+    assert np.array_equal(np.array(firsts, np.int32), x[::512])
+    deltas = np.diff(x.astype(np.int64))
+    rebuilt = np.concatenate([[x[0]], x[0] + np.cumsum(deltas)]).astype(np.int32)
+    assert np.array_equal(oracle.dfor_decode(e), rebuilt)
+
+
+def test_rfor_is_repeat_of_runs():
+    """RLE decode == np.repeat(values, lengths); runs split at 512-row blocks."""
+    x = datagen.runs(512 * 7 + 301, 9, seed=4)
+    out = oracle.rfor_decode(oracle.rfor_encode(x))
+    vals, lens = [], []
+    for k in range(0, len(x), 512):
+        blk = x[k:k + 512]
+        cut = np.flatnonzero(np.diff(blk)) + 1
+        starts = np.concatenate([[0], cut])
+        vals.append(blk[starts])
+        lens.append(np.diff(np.concatenate([starts, [len(blk)]])))
+    assert np.array_equal(out, np.repeat(np.concatenate(vals), np.concatenate(lens)))
+
+
+def test_bitwidth_0_and_32():
+    for x in (np.zeros(1000, np.int32), np.full(1000, -5, np.int32),
+              np.random.default_rng(1).integers(0, 2**32, 1000, dtype=np.uint32).view(np.int32)):
+        for s in ("for", "dfor", "rfor"):
+            assert np.array_equal(oracle.decode(oracle.encode(s, x)), x)
+    e = oracle.for_encode(np.zeros(256, np.int32))
+    assert list(e["starts"]) == [0, 2, 4]          # b = 0 blocks are header only
+
+
+# ---------------------------------------------------------------- golden digests
+def test_golden_rng_free_digests():
+    g = json.load(open(os.path.join(GOLD, "digests.json")))["rng_free"]
+    i = np.arange(1_000_000, dtype=np.int64)
+    j = np.arange(100_000, dtype=np.int64)
+    cols = {"G1": (i * 2**28 // 250_000_000).astype(np.int32),
+            "G2": ((j * j) % 65537 - 32768).astype(np.int32),
+            "G3": (((j // 37) * 2654435761) % 2**32).astype(np.uint32).view(np.int32)}
+    for name, x in cols.items():
+        for s in ("for", "dfor", "rfor"):
+            e = oracle.encode(s, x)
+            assert [e.nbytes(), e.digest()] == g[name][s], (name, s)
+
+
+def test_golden_c1_digests():
+    g = json.load(open(os.path.join(GOLD, "digests.json")))["c1_for"]
+    for b in range(1, 17):
+        x = datagen.c1_column(b)
+        in_digest, size, digest = g[str(b)]
+        if hashlib.sha256(x.tobytes()).hexdigest()[:16] != in_digest:
+            pytest.skip("numpy Generator stream differs from the one the digests were made with")
+        e = oracle.for_encode(x)
+        assert e.nbytes() == size == 4 * (23443 + 31250 * b)
+        assert e.digest() == digest
+
+
+# ---------------------------------------------------------------- queries
+def test_select_project_sum_definition():
+    rng = np.random.default_rng(9)
+    n = 20000
+    a = rng.integers(0, 50, n, dtype=np.int32)
+    b = rng.integers(0, 11, n, dtype=np.int32)
+    c = rng.integers(-(2**31), 2**31, n, dtype=np.int64).astype(np.int32)
+    m = (a >= 1) & (a <= 24) & (b >= 1) & (b <= 3)
+    assert oracle.select_project_sum([a, b, c], [1, 1, -(2**31)], [24, 3, 2**31 - 1], "mul", 2, 1) == \
+        int((c[m].astype(np.int64) * b[m]).sum())
+    assert oracle.select_project_sum([a, b], [0, 0], [49, 10], "sub", 0, 1) == int((a.astype(np.int64) - b).sum())
+    assert oracle.select_project_sum([a], [10, ], [9], "col", 0, 0) == 0
+    assert oracle.column_sum(c) == int(c.astype(np.int64).sum())
+
+
+def test_choose_scheme_gpu_star():
+    """DFOR for sorted high-NDV, RFOR for long runs, FOR for random."""
+    assert oracle.choose_scheme(datagen.d1_prefix(100_000, 2**28, 250_000_000))[0] == "dfor"
+    assert oracle.choose_scheme(datagen.runs(100_000, 32, seed=1))[0] == "rfor"
+    assert oracle.choose_scheme(datagen.uniform_bits(12, 100_000, seed=1))[0] == "for"
