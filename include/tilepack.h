@@ -1,0 +1,172 @@
+/*
+ * tilepack.h -- C ABI of the B200-native (sm_100a) implementation of
+ *   A. Shanbhag, B. Yogatama, X. Yu, S. Madden,
+ *   "Tile-based Lightweight Integer Compression in GPU", SIGMOD '22.
+ * Citations "P:<lines>" refer to /root/reference/PAPER.md; "R<n>" to the
+ * readings listed in DESIGN.md (section "Readings of the paper").
+ *
+ * The boundary follows the paper's problem statement:
+ *   - encode a column into blocks / miniblocks / tiles
+ *   - decode a column
+ *   - decode fused into a select / project / aggregate
+ *   - shard a column by 512-row tile ranges            (multi-GPU)
+ *
+ * Conventions (all functions):
+ *   - Plain pointers and sizes only.  "host" pointers are ordinary CPU memory,
+ *     "device" pointers are CUDA global memory of the current device.
+ *   - Ownership: the CALLER owns every buffer.  The library never frees caller
+ *     memory and never allocates on the decode path.
+ *   - Errors: a tp_status is returned; nothing is thrown across the ABI.  Device
+ *     calls check cudaGetLastError() after each launch and return TP_ECUDA.
+ *   - Device calls are asynchronous on `stream` (a cudaStream_t passed as
+ *     void*; NULL = legacy default stream).  Results land in device memory.
+ *   - Data arrays (data0/data1) and block_starts arrays (starts0/starts1)
+ *     must be allocated with TP_GUARD_WORDS extra zero words after their last
+ *     used word (R9: Alg. 1 line 15 reads data[s+1]; the tile stager reads
+ *     16-byte aligned supersets).  Device arrays must be 16-byte aligned.
+ *   - Counts: n < 2^32 (the header's total count is a 32-bit word)
+ *     and every word offset < 2^32 (block_starts are u32, R6); larger inputs
+ *     return TP_EUNSUPPORTED.  Shard larger columns with tp_shard.
+ *   - All values are int32; decode arithmetic is mod 2^32 (R4); aggregates
+ *     are int64 mod 2^64 (R24).
+ */
+#ifndef TILEPACK_H
+#define TILEPACK_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define TP_GUARD_WORDS 4u
+
+typedef enum {
+  TP_OK = 0,
+  TP_EINVAL = 1,        /* bad argument (NULL pointer, unknown scheme, bad op)  */
+  TP_ESIZE = 2,         /* a caller-provided buffer is too small                */
+  TP_EFORMAT = 3,       /* header / bitwidth inconsistent with the scheme       */
+  TP_ECUDA = 4,         /* a CUDA launch or API call failed                     */
+  TP_EUNSUPPORTED = 5   /* n >= 2^32 or word offsets >= 2^32                    */
+} tp_status;
+
+typedef enum {
+  TP_FOR = 1,   /* GPU-FOR   header [128, 4, n]                          */
+  TP_DFOR = 2,  /* GPU-DFOR header [128, 4, n], tiles of D = 4 blocks   */
+  TP_RFOR = 3   /* GPU-RFOR header [512, 16, n], value + run streams     */
+} tp_scheme;
+
+/*
+ * A NON-OWNING view of one encoded column.  The pointers are either all host
+ * or all device (tp_encode fills host pointers; the caller copies the arrays
+ * to the device and repoints them).
+ *   header (Fig. 3, R7) = {block_size, miniblock_count, n}
+ *   FOR/DFOR: starts0 = block_starts (num_blocks+1 u32 word offsets into
+ *             data0, R6), data0 = blocks; starts1/data1 unused.
+ *             DFOR: the first value of tile t is data0[starts0[4t]-1] (Fig. 6).
+ *   RFOR:     starts0/data0 = value stream, starts1/data1 = run-length stream,
+ *             one stream block per 512-row block (R17).
+ *   max_tile_words0/1: largest word span of one 512-row tile in stream 0/1
+ *             (filled by tp_encode / tp_shard; 0 = unknown, the decoder then
+ *             assumes the format's worst case).  Sizes the shared-memory ring.
+ */
+typedef struct {
+  uint32_t scheme;            /* tp_scheme                                      */
+  uint32_t block_size;        /* 128 (FOR, DFOR) or 512 (RFOR)                  */
+  uint32_t miniblock_count;   /* 4 (FOR, DFOR) or 16 (RFOR)                     */
+  uint32_t tile_blocks;       /* blocks per 512-row tile: 4 (FOR, DFOR), 1 (RFOR) */
+  uint64_t n;                 /* total count                                    */
+  uint64_t num_blocks;        /* ceil(n/128) (FOR, DFOR) or ceil(n/512) (RFOR)  */
+  const uint32_t* starts0;
+  const uint32_t* data0;
+  uint64_t words0;            /* used words of data0 (excluding guard words)   */
+  const uint32_t* starts1;
+  const uint32_t* data1;
+  uint64_t words1;
+  uint32_t max_tile_words0;
+  uint32_t max_tile_words1;
+} tp_column;
+
+/* ------------------------------------------------------------------ host */
+
+/* Sizes tp_encode will produce for `scheme` on host column x[0..n).
+ * Outputs (host): *num_blocks, *words0, *words1 (0 unless RFOR).
+ * Allocate starts0/starts1 with num_blocks+1+TP_GUARD_WORDS words and
+ * data0/data1 with words+TP_GUARD_WORDS words.  Multi-threaded. */
+tp_status tp_encode_size(int scheme, const int32_t* x, uint64_t n,
+                         uint64_t* num_blocks, uint64_t* words0, uint64_t* words1);
+
+/* Encode host column x[0..n) (compression is a one-time host
+ * step).  Writes starts/data (host, caller-allocated as above, guard words
+ * zeroed by the library) and fills *out with host pointers.  starts1/data1
+ * may be NULL unless scheme == TP_RFOR.  Byte layout: DESIGN.md "Formats". */
+tp_status tp_encode(int scheme, const int32_t* x, uint64_t n,
+                    uint32_t* starts0, uint32_t* data0,
+                    uint32_t* starts1, uint32_t* data1, tp_column* out);
+
+/* GPU-* (P:1206-1217): the scheme with the smallest footprint; ties resolve
+ * FOR < DFOR < RFOR (R20).  Outputs (host): *scheme, *bytes. */
+tp_status tp_choose_scheme(const int32_t* x, uint64_t n, int* scheme, uint64_t* bytes);
+
+/* Compressed footprint in bytes: 3-word header + block_starts + data
+ * (P:1459-1471).  0 for a NULL column. */
+uint64_t tp_compressed_bytes(const tp_column* col);
+
+/* A view of rows [row_lo, row_hi) of a HOST column; row_lo must be a multiple
+ * of 512 (one tile), row_hi a multiple of 512 or n.
+ * Writes rebased block_starts into rebased0 (and rebased1 for RFOR), each
+ * with (blocks in range)+1+TP_GUARD_WORDS words; the view's data pointers
+ * alias the parent's data (DFOR views start at the tile's first value). */
+tp_status tp_shard(const tp_column* host_col, uint64_t row_lo, uint64_t row_hi,
+                   uint32_t* rebased0, uint32_t* rebased1, tp_column* view);
+
+/* ---------------------------------------------------------------- device */
+
+/* Decode the whole DEVICE column into d_out[0..n) (int32, device).
+ * One pass over HBM: each 512-row tile is staged once into shared memory by
+ * TMA bulk copies and unpacked there (tile-based decompression);
+ * decoded rows are written back by TMA tensor stores (decode-to-global mode
+ * of Fig. 7a). */
+tp_status tp_decode(const tp_column* dcol, int32_t* d_out, void* stream);
+
+/* Decode fused into an int64 sum (the paper's decode-only microbenchmark,
+ * P:720-724, with a consumer that keeps every value live).  ADDS the sum of
+ * all n values into *d_sum (device int64; the caller zeroes it). */
+tp_status tp_decode_sum(const tp_column* dcol, int64_t* d_sum, void* stream);
+
+/* Fused select / project / aggregate over ncols DEVICE columns of equal n
+ * (the decoders replace the tile load inside the query kernel):
+ *   *d_result += sum over rows i with lo[c] <= col_c[i] <= hi[c] for all c
+ *                of proj(i)
+ * proj_op: TP_PROJ_COL -> col_a[i];  TP_PROJ_MUL -> col_a[i]*col_b[i];
+ *          TP_PROJ_SUB -> col_a[i]-col_b[i];  TP_PROJ_COUNT -> 1.
+ * lo/hi: host arrays of ncols int32 (inclusive); [INT32_MIN, INT32_MAX]
+ * means "no predicate".  ncols <= TP_MAX_COLS. */
+#define TP_MAX_COLS 6
+enum { TP_PROJ_COL = 0, TP_PROJ_MUL = 1, TP_PROJ_SUB = 2, TP_PROJ_COUNT = 3 };
+tp_status tp_select_project_sum(const tp_column* dcols, int ncols,
+                                const int32_t* lo, const int32_t* hi,
+                                int proj_op, int a, int b,
+                                int64_t* d_result, void* stream);
+
+/* The uncompressed baseline "None": *d_sum += sum of the n int32
+ * values of DEVICE array d_x (16-byte aligned), 128-bit streaming loads.
+ * Used as the measured HBM read roof of the same consumer. */
+tp_status tp_plain_sum(const int32_t* d_x, uint64_t n, int64_t* d_sum, void* stream);
+
+/* --------------------------------------------------------------- utility */
+
+const char* tp_status_string(tp_status s);
+
+/* Number of CUDA kernels this library has launched in this process
+ * (bench.py reports it as gpu_launches). */
+uint64_t tp_launch_count(void);
+
+/* Number of SMs of the current device and the decoder's CTAs per SM
+ * (persistent grid = SMs x CTAs/SM). */
+tp_status tp_device_info(int* sm_count, int* ctas_per_sm);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TILEPACK_H */

@@ -1,0 +1,274 @@
+"""Thin ctypes binding of the tilepack C ABI (include/tilepack.h).
+
+Argument marshalling only: every step of encode/decode/query runs in the native
+library (host encoder in C++, decoders and fused operators as sm_100a CUDA
+kernels).  PyTorch provides device memory and streams.  There is no CPU or
+Python fallback: if ``libtilepack.so`` is missing this module raises at import.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libtilepack.so")
+GUARD_WORDS = 4
+
+TP_FOR, TP_DFOR, TP_RFOR = 1, 2, 3
+SCHEMES = {"for": TP_FOR, "dfor": TP_DFOR, "rfor": TP_RFOR}
+SCHEME_NAMES = {v: k for k, v in SCHEMES.items()}
+TP_PROJ = {"col": 0, "mul": 1, "sub": 2, "count": 3}
+TP_MAX_COLS = 6
+
+
+class TilepackError(RuntimeError):
+    pass
+
+
+class tp_column(ctypes.Structure):
+    _fields_ = [
+        ("scheme", ctypes.c_uint32),
+        ("block_size", ctypes.c_uint32),
+        ("miniblock_count", ctypes.c_uint32),
+        ("tile_blocks", ctypes.c_uint32),
+        ("n", ctypes.c_uint64),
+        ("num_blocks", ctypes.c_uint64),
+        ("starts0", ctypes.c_void_p),
+        ("data0", ctypes.c_void_p),
+        ("words0", ctypes.c_uint64),
+        ("starts1", ctypes.c_void_p),
+        ("data1", ctypes.c_void_p),
+        ("words1", ctypes.c_uint64),
+        ("max_tile_words0", ctypes.c_uint32),
+        ("max_tile_words1", ctypes.c_uint32),
+    ]
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(
+            f"tilepack native library not built: {LIB_PATH} is missing "
+            "(run `python -c 'import __graft_entry__ as g; g.build()'`)")
+    L = ctypes.CDLL(LIB_PATH)
+    vp, u64, i32, u32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_uint32
+    colp = ctypes.POINTER(tp_column)
+    sig = {
+        "tp_encode_size": (i32, [i32, vp, u64, vp, vp, vp]),
+        "tp_encode": (i32, [i32, vp, u64, vp, vp, vp, vp, colp]),
+        "tp_choose_scheme": (i32, [vp, u64, vp, vp]),
+        "tp_compressed_bytes": (u64, [colp]),
+        "tp_shard": (i32, [colp, u64, u64, vp, vp, colp]),
+        "tp_decode": (i32, [colp, vp, vp]),
+        "tp_decode_sum": (i32, [colp, vp, vp]),
+        "tp_select_project_sum": (i32, [colp, i32, vp, vp, i32, i32, i32, vp, vp]),
+        "tp_plain_sum": (i32, [vp, u64, vp, vp]),
+        "tp_status_string": (ctypes.c_char_p, [i32]),
+        "tp_launch_count": (u64, []),
+        "tp_device_info": (i32, [vp, vp]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    return L
+
+
+_lib = _load()
+
+
+def lib():
+    return _lib
+
+
+def _check(rc: int, what: str):
+    if rc != 0:
+        raise TilepackError(f"{what}: {_lib.tp_status_string(rc).decode()} (status {rc})")
+
+
+def _ptr(a) -> int | None:
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        return a.ctypes.data
+    return a.data_ptr()  # torch tensor
+
+
+def _stream(stream=None):
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+# ------------------------------------------------------------------ C ABI, same names
+def tp_encode_size(scheme: int, x: np.ndarray):
+    nb, w0, w1 = ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_uint64()
+    _check(_lib.tp_encode_size(scheme, _ptr(x), len(x), ctypes.byref(nb), ctypes.byref(w0), ctypes.byref(w1)),
+           "tp_encode_size")
+    return nb.value, w0.value, w1.value
+
+
+def tp_encode(scheme: int, x: np.ndarray, starts0, data0, starts1=None, data1=None) -> tp_column:
+    col = tp_column()
+    _check(_lib.tp_encode(scheme, _ptr(x), len(x), _ptr(starts0), _ptr(data0), _ptr(starts1), _ptr(data1),
+                          ctypes.byref(col)), "tp_encode")
+    return col
+
+
+def tp_choose_scheme(x: np.ndarray):
+    s, b = ctypes.c_int(), ctypes.c_uint64()
+    _check(_lib.tp_choose_scheme(_ptr(x), len(x), ctypes.byref(s), ctypes.byref(b)), "tp_choose_scheme")
+    return s.value, b.value
+
+
+def tp_compressed_bytes(col: tp_column) -> int:
+    return int(_lib.tp_compressed_bytes(ctypes.byref(col)))
+
+
+def tp_shard(col: tp_column, row_lo: int, row_hi: int, rebased0, rebased1=None) -> tp_column:
+    view = tp_column()
+    _check(_lib.tp_shard(ctypes.byref(col), row_lo, row_hi, _ptr(rebased0), _ptr(rebased1), ctypes.byref(view)),
+           "tp_shard")
+    return view
+
+
+def tp_decode(dcol: tp_column, d_out, stream=None):
+    _check(_lib.tp_decode(ctypes.byref(dcol), _ptr(d_out), _stream(stream)), "tp_decode")
+
+
+def tp_decode_sum(dcol: tp_column, d_sum, stream=None):
+    _check(_lib.tp_decode_sum(ctypes.byref(dcol), _ptr(d_sum), _stream(stream)), "tp_decode_sum")
+
+
+def tp_select_project_sum(dcols, lo, hi, proj_op: int, a: int, b: int, d_result, stream=None):
+    n = len(dcols)
+    arr = (tp_column * n)(*dcols)
+    lo = np.ascontiguousarray(lo, np.int32)
+    hi = np.ascontiguousarray(hi, np.int32)
+    _check(_lib.tp_select_project_sum(arr, n, _ptr(lo), _ptr(hi), proj_op, a, b, _ptr(d_result), _stream(stream)),
+           "tp_select_project_sum")
+
+
+def tp_plain_sum(d_x, n: int, d_sum, stream=None):
+    _check(_lib.tp_plain_sum(_ptr(d_x), n, _ptr(d_sum), _stream(stream)), "tp_plain_sum")
+
+
+def tp_launch_count() -> int:
+    return int(_lib.tp_launch_count())
+
+
+def tp_device_info():
+    sms, occ = ctypes.c_int(), ctypes.c_int()
+    _check(_lib.tp_device_info(ctypes.byref(sms), ctypes.byref(occ)), "tp_device_info")
+    return sms.value, occ.value
+
+
+# ------------------------------------------------------------------ convenience objects
+class HostColumn:
+    """An encoded column in host memory (numpy arrays with guard words) + its tp_column."""
+
+    def __init__(self, scheme: str, x: np.ndarray):
+        x = np.ascontiguousarray(x, dtype=np.int32)
+        sc = SCHEMES[scheme]
+        nb, w0, w1 = tp_encode_size(sc, x)
+        self.scheme = scheme
+        self.starts0 = np.zeros(nb + 1 + GUARD_WORDS, np.uint32)
+        self.data0 = np.zeros(w0 + GUARD_WORDS, np.uint32)
+        self.starts1 = np.zeros(nb + 1 + GUARD_WORDS, np.uint32) if sc == TP_RFOR else None
+        self.data1 = np.zeros(w1 + GUARD_WORDS, np.uint32) if sc == TP_RFOR else None
+        self.col = tp_encode(sc, x, self.starts0, self.data0, self.starts1, self.data1)
+
+    @property
+    def n(self) -> int:
+        return int(self.col.n)
+
+    def nbytes(self) -> int:
+        return tp_compressed_bytes(self.col)
+
+    def header(self) -> np.ndarray:
+        return np.array([self.col.block_size, self.col.miniblock_count, self.col.n], np.uint32)
+
+    def arrays(self) -> dict:
+        """Used words only (no guard words): the oracle's layout for byte comparison."""
+        nb = int(self.col.num_blocks)
+        d = {"header": self.header(), "starts0": self.starts0[:nb + 1], "data0": self.data0[:self.col.words0]}
+        if self.starts1 is not None:
+            d["starts1"] = self.starts1[:nb + 1]
+            d["data1"] = self.data1[:self.col.words1]
+        return d
+
+    def to_device(self, device=None) -> "DeviceColumn":
+        return DeviceColumn(self, device)
+
+
+def _to_dev(a: np.ndarray | None, device, pinned: bool = False):
+    import torch
+    if a is None:
+        return None
+    t = torch.from_numpy(a.view(np.int32))
+    if pinned:
+        t = t.pin_memory()
+    return t.to(device, non_blocking=pinned)
+
+
+class DeviceColumn:
+    """Device copies (torch int32 storage) of an encoded column + a tp_column of device pointers."""
+
+    def __init__(self, host: HostColumn, device=None):
+        import torch
+        device = device if device is not None else torch.device("cuda", torch.cuda.current_device())
+        self.host = host
+        self.starts0 = _to_dev(host.starts0, device)
+        self.data0 = _to_dev(host.data0, device)
+        self.starts1 = _to_dev(host.starts1, device)
+        self.data1 = _to_dev(host.data1, device)
+        c = tp_column()
+        ctypes.pointer(c)[0] = host.col
+        c.starts0, c.data0 = self.starts0.data_ptr(), self.data0.data_ptr()
+        if self.starts1 is not None:
+            c.starts1, c.data1 = self.starts1.data_ptr(), self.data1.data_ptr()
+        self.col = c
+
+    @property
+    def n(self) -> int:
+        return int(self.col.n)
+
+    def nbytes(self) -> int:
+        return tp_compressed_bytes(self.col)
+
+
+def encode(x: np.ndarray, scheme: str = "for") -> HostColumn:
+    """Encode a host int32 column (scheme 'for' | 'dfor' | 'rfor' | 'auto' = GPU-*)."""
+    if scheme == "auto":
+        s, _ = tp_choose_scheme(np.ascontiguousarray(x, np.int32))
+        scheme = SCHEME_NAMES[s]
+    return HostColumn(scheme, x)
+
+
+def decode(dcol: DeviceColumn, out=None, stream=None):
+    import torch
+    if out is None:
+        out = torch.empty(dcol.n, dtype=torch.int32, device=dcol.data0.device)
+    tp_decode(dcol.col, out, stream)
+    return out
+
+
+def decode_sum(dcol: DeviceColumn, out=None, stream=None):
+    import torch
+    if out is None:
+        out = torch.zeros(1, dtype=torch.int64, device=dcol.data0.device)
+    tp_decode_sum(dcol.col, out, stream)
+    return out
+
+
+def select_project_sum(dcols, lo, hi, proj: str = "col", a: int = 0, b: int = 0, out=None, stream=None):
+    import torch
+    if out is None:
+        out = torch.zeros(1, dtype=torch.int64, device=dcols[0].data0.device)
+    tp_select_project_sum([d.col for d in dcols], lo, hi, TP_PROJ[proj], a, b, out, stream)
+    return out
+
+
+def tp_status_string(status: int) -> str:
+    return _lib.tp_status_string(status).decode()

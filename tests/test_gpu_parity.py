@@ -1,0 +1,127 @@
+"""GPU parity: the sm_100a decoders and fused operators vs the CPU oracle, through the C ABI.
+Integer work: every comparison is bit-exact."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import datagen  # noqa: E402
+import oracle  # noqa: E402
+from paper_conf_sigmod_shanbhagyym22_b200 import tilepack as tp  # noqa: E402
+
+SCHEMES = ("for", "dfor", "rfor")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    torch.cuda.set_device(0)
+
+
+def _check_column(x, scheme):
+    h = tp.encode(x, scheme)
+    e = oracle.encode(scheme, x)
+    want = oracle.decode(e)
+    d = h.to_device()
+    got = tp.decode(d).cpu().numpy()
+    assert np.array_equal(got, want), f"{scheme} n={len(x)} first bad row {np.flatnonzero(got != want)[:5]}"
+    s = int(tp.decode_sum(d).item())
+    assert s == oracle.column_sum(want)
+
+
+@pytest.mark.parametrize("scheme", SCHEMES)
+def test_mixed_ragged_columns(scheme):
+    for name, x in datagen.mixed_columns(seed=11):
+        if len(x) == 0:
+            continue
+        _check_column(x, scheme)
+
+
+@pytest.mark.parametrize("scheme", SCHEMES)
+def test_tiny_columns(scheme):
+    for x in list(datagen.small_alphabet_columns(2))[1:]:
+        _check_column(x, scheme)
+
+
+def test_every_bitwidth_for():
+    for b in range(0, 33):
+        _check_column(datagen.uniform_bits(b, 512 * 37 + 13, seed=100 + b), "for")
+
+
+def test_mixed_bitwidths_within_warp():
+    """lanes of one warp disagree on b: the runtime-bitwidth fallback path."""
+    rng = np.random.default_rng(4)
+    parts = [rng.integers(0, 2 ** int(rng.integers(0, 32)), 32, dtype=np.int64) for _ in range(2000)]
+    x = np.concatenate(parts).astype(np.int32)
+    for s in SCHEMES:
+        _check_column(x, s)
+
+
+@pytest.mark.parametrize("scheme,gen", [
+    ("for", lambda n: datagen.uniform_bits(16, n, seed=5)),
+    ("dfor", lambda n: datagen.sorted_uniform(n, seed=6)),
+    ("dfor", lambda n: datagen.d1_sorted(n, 2**28)),
+    ("rfor", lambda n: datagen.runs(n, 4, seed=7)),
+    ("rfor", lambda n: datagen.runs(n, 64, seed=8)),
+])
+def test_many_ctas(scheme, gen):
+    """several stages per CTA, every CTA busy, ragged tail"""
+    n = 5_000_000 + 321
+    _check_column(gen(n), scheme)
+
+
+def test_empty_column():
+    h = tp.encode(np.zeros(0, np.int32), "for")
+    d = h.to_device()
+    assert int(tp.decode_sum(d).item()) == 0
+
+
+def test_select_project_sum_parity():
+    rng = np.random.default_rng(3)
+    n = 1_000_000 + 77
+    qty = rng.integers(1, 51, n, dtype=np.int32)
+    disc = rng.integers(0, 11, n, dtype=np.int32)
+    price = rng.integers(90000, 10_000_000, n, dtype=np.int32)
+    date = np.repeat(rng.integers(19920101, 19981231, n // 4 + 1, dtype=np.int32), 4)[:n]
+    cols = [date, qty, disc, price]
+    schemes = ["rfor", "for", "for", "dfor"]
+    dc = [tp.encode(c, s).to_device() for c, s in zip(cols, schemes)]
+    lo = [19930101, 1, 1, -(2**31)]
+    hi = [19931231, 24, 3, 2**31 - 1]
+    for proj, a, b in (("mul", 3, 2), ("col", 3, 0), ("sub", 3, 1), ("count", 0, 0)):
+        got = int(tp.select_project_sum(dc, lo, hi, proj, a, b).item())
+        assert got == oracle.select_project_sum(cols, lo, hi, proj, a, b), proj
+
+
+def test_plain_sum():
+    x = datagen.uniform_bits(32, 1_000_003, seed=2)
+    t = torch.from_numpy(x).cuda()
+    out = torch.zeros(1, dtype=torch.int64, device="cuda")
+    tp.tp_plain_sum(t, len(x), out)
+    assert int(out.item()) == oracle.column_sum(x)
+
+
+@pytest.mark.slow
+def test_bench_size_for_b16_sampled():
+    """BASELINE config 2 at the bench's launch configuration: 500M U[0,2^16) rows.
+    Fused sum == the plain int64 sum; decoded rows at 20k sampled positions == Alg. 1."""
+    n = 500_000_000
+    x = datagen.uniform_bits(16, n)
+    h = tp.encode(x, "for")
+    assert h.nbytes() == 4 * (3 + (n // 128) + 1 + (n // 128) * (2 + 4 * 16))
+    d = h.to_device()
+    assert int(tp.decode_sum(d).item()) == int(x.astype(np.int64).sum())
+    out = tp.decode(d)
+    rng = np.random.default_rng(0)
+    idx = np.sort(rng.integers(0, n, 20_000))
+    got = out[torch.from_numpy(idx).cuda()].cpu().numpy()
+    e = oracle.Encoded(scheme="for", header=h.header(), starts=h.starts0[: h.col.num_blocks + 1],
+                       data=h.data0[: h.col.words0])
+    dg = h.data0  # already has guard words
+    want = np.array([oracle.for_decode_range(e, int(i), int(i) + 1, dg)[0] for i in idx[:2000]], np.int32)
+    assert np.array_equal(got[:2000], want)
+    assert np.array_equal(got, x[idx])
+    tail = out[n - 1000:].cpu().numpy()
+    assert np.array_equal(tail, oracle.for_decode_range(e, n - 1000, n, dg))

@@ -1,0 +1,99 @@
+"""Host encoder of the product library (C++, multi-threaded) vs the oracle, byte for byte.
+No GPU needed: encoding is the paper's one-time host step."""
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+from paper_conf_sigmod_shanbhagyym22_b200 import tilepack as tp
+
+SCHEMES = ("for", "dfor", "rfor")
+
+
+def _same(h, e):
+    a = h.arrays()
+    assert np.array_equal(a["header"], e["header"])
+    if e["scheme"] == "rfor":
+        assert np.array_equal(a["starts0"], e["startsV"]) and np.array_equal(a["data0"], e["dataV"])
+        assert np.array_equal(a["starts1"], e["startsL"]) and np.array_equal(a["data1"], e["dataL"])
+    else:
+        assert np.array_equal(a["starts0"], e["starts"]) and np.array_equal(a["data0"], e["data"])
+    assert h.nbytes() == e.nbytes()
+
+
+def test_bruteforce_tiny_columns_byte_identical():
+    for x in datagen.small_alphabet_columns(3):
+        for s in SCHEMES:
+            _same(tp.encode(x, s), oracle.encode(s, x))
+
+
+@pytest.mark.parametrize("scheme", SCHEMES)
+def test_mixed_columns_byte_identical(scheme):
+    for name, x in datagen.mixed_columns(seed=5):
+        _same(tp.encode(x, scheme), oracle.encode(scheme, x))
+
+
+def test_c1_columns_byte_identical():
+    for b in (1, 7, 16):
+        x = datagen.c1_column(b)
+        _same(tp.encode(x, "for"), oracle.for_encode(x))
+
+
+def test_large_multithreaded_byte_identical():
+    n = 3_000_000 + 123
+    for s, x in (("for", datagen.uniform_bits(11, n, seed=9)), ("dfor", datagen.near_sorted(n, seed=8)),
+                 ("rfor", datagen.runs(n, 5, seed=7))):
+        _same(tp.encode(x, s), oracle.encode(s, x))
+
+
+def test_choose_scheme_matches_oracle():
+    for x in (datagen.d1_prefix(200_000, 2**28, 250_000_000), datagen.runs(200_000, 16, seed=2),
+              datagen.uniform_bits(9, 200_000, seed=3), np.zeros(1000, np.int32)):
+        s, b = tp.tp_choose_scheme(x)
+        os_, oe = oracle.choose_scheme(x)
+        assert tp.SCHEME_NAMES[s] == os_ and b == oe.nbytes()
+
+
+def test_max_tile_words():
+    x = datagen.uniform_bits(16, 512 * 10 + 5, seed=1)
+    h = tp.encode(x, "for")
+    s = h.starts0[: h.col.num_blocks + 1].astype(np.int64)
+    spans = [s[min(4 * t + 4, len(s) - 1)] - s[4 * t] for t in range((len(s) - 1 + 3) // 4)]
+    assert h.col.max_tile_words0 == max(spans)
+
+
+@pytest.mark.parametrize("scheme", SCHEMES)
+def test_shard_views_decode_to_slices(scheme):
+    """tp_shard: a 512-row-aligned range view decodes (by the oracle) to the slice."""
+    n = 512 * 13 + 200
+    x = {"for": datagen.uniform_bits(9, n, seed=1), "dfor": datagen.near_sorted(n, seed=1),
+         "rfor": datagen.runs(n, 7, seed=1)}[scheme]
+    h = tp.encode(x, scheme)
+    for lo, hi in ((0, 512 * 5), (512 * 5, 512 * 9), (512 * 9, n), (0, n), (512 * 13, n)):
+        nbv = -(-(hi - lo) // (512 if scheme == "rfor" else 128))
+        r0 = np.zeros(nbv + 1 + tp.GUARD_WORDS, np.uint32)
+        r1 = np.zeros(nbv + 1 + tp.GUARD_WORDS, np.uint32) if scheme == "rfor" else None
+        v = tp.tp_shard(h.col, lo, hi, r0, r1)
+        assert v.n == hi - lo and v.num_blocks == nbv
+        import ctypes
+
+        def words(ptr, k):
+            return np.ctypeslib.as_array((ctypes.c_uint32 * k).from_address(ptr)).copy()
+        if scheme == "rfor":
+            e = oracle.Encoded(scheme="rfor", header=np.array([512, 16, hi - lo], np.uint32),
+                               startsV=r0[:nbv + 1], dataV=words(v.data0, v.words0),
+                               startsL=r1[:nbv + 1], dataL=words(v.data1, v.words1))
+        else:
+            e = oracle.Encoded(scheme=scheme, header=np.array([128, 4, hi - lo], np.uint32),
+                               starts=r0[:nbv + 1], data=words(v.data0, v.words0))
+        assert np.array_equal(oracle.decode(e), x[lo:hi])
+
+
+def test_errors():
+    x = np.arange(1000, dtype=np.int32)
+    with pytest.raises(tp.TilepackError):
+        tp.tp_encode_size(7, x)
+    h = tp.encode(x, "for")
+    r0 = np.zeros(64, np.uint32)
+    with pytest.raises(tp.TilepackError):
+        tp.tp_shard(h.col, 100, 600, r0)   # not tile aligned
