@@ -1,0 +1,110 @@
+"""Seeded SSB-shaped data (Star Schema Benchmark [35], used at SF 20 in P:1874-1888).
+
+Holds no compression arithmetic.  String attributes are emitted directly as dictionary
+codes with the mapping of SURVEY.md Appendix B:
+  region 0..4 (AFRICA, AMERICA, ASIA, EUROPE, MIDDLE EAST); nation 0..24 (TPC-H order,
+  NATION_REGION below); city = nation*10 + digit ('UNITED KI1' = 231);
+  p_mfgr m in 1..5; p_category = 10m + c, c in 1..5 ('MFGR#12' = 12);
+  p_brand1 = 100*category + k, k in 1..40 ('MFGR#2221' = 2221);
+  d_datekey = yyyymmdd, d_yearmonthnum = d_yearmonth = yyyymm, d_weeknuminyear = (doy-1)//7 + 1.
+Lineorder keeps the dbgen run structure that decides GPU-* (P:1916-1918): orders of 1..7
+lines, orderdate / custkey / orderpriority constant per order.
+"""
+from __future__ import annotations
+
+import datetime as _dt
+import math
+
+import numpy as np
+
+REGIONS = ["AFRICA", "AMERICA", "ASIA", "EUROPE", "MIDDLE EAST"]
+NATIONS = ["ALGERIA", "ARGENTINA", "BRAZIL", "CANADA", "EGYPT", "ETHIOPIA", "FRANCE", "GERMANY", "INDIA",
+           "INDONESIA", "IRAN", "IRAQ", "JAPAN", "JORDAN", "KENYA", "MOROCCO", "MOZAMBIQUE", "PERU", "CHINA",
+           "ROMANIA", "SAUDI ARABIA", "VIETNAM", "RUSSIA", "UNITED KINGDOM", "UNITED STATES"]
+NATION_REGION = np.array([0, 1, 1, 1, 4, 0, 3, 3, 2, 2, 4, 4, 2, 4, 0, 0, 0, 1, 2, 3, 4, 2, 3, 3, 1], np.int32)
+AMERICA, ASIA, EUROPE = 1, 2, 3
+UNITED_STATES, UNITED_KINGDOM = 24, 23
+
+LINEORDER_COLUMNS = ("lo_orderkey", "lo_linenumber", "lo_custkey", "lo_partkey", "lo_suppkey", "lo_orderdate",
+                     "lo_orderpriority", "lo_quantity", "lo_extendedprice", "lo_ordtotalprice", "lo_discount",
+                     "lo_revenue", "lo_supplycost", "lo_tax", "lo_commitdate")
+QUERY_COLUMNS = ("lo_orderdate", "lo_quantity", "lo_discount", "lo_extendedprice", "lo_partkey", "lo_suppkey",
+                 "lo_revenue", "lo_custkey", "lo_supplycost")
+
+
+def sizes(sf: float) -> dict:
+    return {"customer": int(30_000 * sf), "supplier": int(2_000 * sf),
+            "part": int(200_000 * math.floor(1 + math.log2(sf))) if sf >= 1 else int(200_000 * sf),
+            "orders": int(1_500_000 * sf)}
+
+
+def date_dim() -> dict:
+    """1992-01-01 .. 1998-12-31 (the SSB date dimension, 7 years)."""
+    d0 = _dt.date(1992, 1, 1)
+    days = (_dt.date(1998, 12, 31) - d0).days + 1
+    keys, year, ym, week = [], [], [], []
+    for i in range(days):
+        d = d0 + _dt.timedelta(days=i)
+        keys.append(d.year * 10000 + d.month * 100 + d.day)
+        year.append(d.year)
+        ym.append(d.year * 100 + d.month)
+        week.append((d.timetuple().tm_yday - 1) // 7 + 1)
+    a = lambda v: np.array(v, np.int32)  # noqa: E731
+    return {"d_datekey": a(keys), "d_year": a(year), "d_yearmonthnum": a(ym), "d_yearmonth": a(ym),
+            "d_weeknuminyear": a(week)}
+
+
+def generate(sf: float, seed: int = 5000) -> dict:
+    """Returns {'lineorder': {col: int32 array}, 'date': ..., 'customer': ..., 'supplier': ..., 'part': ...}."""
+    rng = np.random.default_rng(seed)
+    z = sizes(sf)
+    C, S, P, O = z["customer"], z["supplier"], z["part"], z["orders"]
+    date = date_dim()
+    # dimensions (keys are dense 1..N; attributes uniform like dbgen)
+    c_nation = rng.integers(0, 25, C, dtype=np.int32)
+    customer = {"c_custkey": np.arange(1, C + 1, dtype=np.int32), "c_nation": c_nation,
+                "c_region": NATION_REGION[c_nation], "c_city": c_nation * 10 + rng.integers(0, 10, C, dtype=np.int32)}
+    s_nation = rng.integers(0, 25, S, dtype=np.int32)
+    supplier = {"s_suppkey": np.arange(1, S + 1, dtype=np.int32), "s_nation": s_nation,
+                "s_region": NATION_REGION[s_nation], "s_city": s_nation * 10 + rng.integers(0, 10, S, dtype=np.int32)}
+    mfgr = rng.integers(1, 6, P, dtype=np.int32)
+    cat = mfgr * 10 + rng.integers(1, 6, P, dtype=np.int32)
+    brand = cat * 100 + rng.integers(1, 41, P, dtype=np.int32)
+    pk = np.arange(1, P + 1, dtype=np.int64)
+    retail = (90000 + (pk // 10) % 20001 + 100 * (pk % 1000)).astype(np.int64)  # TPC-H p_retailprice (cents)
+    part = {"p_partkey": pk.astype(np.int32), "p_mfgr": mfgr, "p_category": cat, "p_brand1": brand}
+    # orders: 1..7 lines, date in [1992-01-01, 1998-08-02], custkey, priority constant per order
+    lines = rng.integers(1, 8, O, dtype=np.int64)
+    n = int(lines.sum())
+    okey = np.arange(1, O + 1, dtype=np.int64)
+    okey = (okey // 8) * 32 + okey % 8                      # sparse TPC-H-style order keys
+    last = int(np.searchsorted(date["d_datekey"], 19980802)) + 1
+    odate = date["d_datekey"][rng.integers(0, last, O)]
+    ocust = rng.integers(1, C + 1, O, dtype=np.int32)
+    oprio = rng.integers(1, 6, O, dtype=np.int32)
+    rep = lambda v: np.repeat(v, lines)  # noqa: E731
+    lo_orderkey = rep(okey).astype(np.int32)
+    starts = np.cumsum(lines) - lines
+    lo_linenumber = (np.arange(n, dtype=np.int64) - rep(starts) + 1).astype(np.int32)
+    qty = rng.integers(1, 51, n, dtype=np.int64)
+    disc = rng.integers(0, 11, n, dtype=np.int64)
+    tax = rng.integers(0, 9, n, dtype=np.int64)
+    lo_partkey = rng.integers(1, P + 1, n, dtype=np.int64)
+    lo_suppkey = rng.integers(1, S + 1, n, dtype=np.int32)
+    ext = qty * retail[lo_partkey - 1]
+    rev = ext * (100 - disc) // 100
+    supplycost = rng.integers(100, 100_001, n, dtype=np.int64)
+    otot = np.bincount(np.repeat(np.arange(O), lines), weights=rev, minlength=O).astype(np.int64)
+    lo_orderdate = rep(odate).astype(np.int32)
+    dayidx = np.searchsorted(date["d_datekey"], lo_orderdate)
+    commit = date["d_datekey"][np.minimum(dayidx + rng.integers(30, 91, n), len(date["d_datekey"]) - 1)]
+    lineorder = {
+        "lo_orderkey": lo_orderkey, "lo_linenumber": lo_linenumber, "lo_custkey": rep(ocust).astype(np.int32),
+        "lo_partkey": lo_partkey.astype(np.int32), "lo_suppkey": lo_suppkey, "lo_orderdate": lo_orderdate,
+        "lo_orderpriority": rep(oprio).astype(np.int32), "lo_quantity": qty.astype(np.int32),
+        "lo_extendedprice": ext.astype(np.int32), "lo_ordtotalprice": np.minimum(rep(otot), 2**31 - 1).astype(np.int32),
+        "lo_discount": disc.astype(np.int32), "lo_revenue": rev.astype(np.int32),
+        "lo_supplycost": supplycost.astype(np.int32), "lo_tax": tax.astype(np.int32),
+        "lo_commitdate": commit.astype(np.int32)}
+    return {"sf": sf, "lineorder": lineorder, "date": date, "customer": customer, "supplier": supplier,
+            "part": part}

@@ -5,7 +5,7 @@
 //
 // Execution model:
 //   * persistent CTAs, one contiguous range of 512-row tiles each;
-//   * warp 0 is a TMA producer: per stage of TPS tiles it issues 1-D bulk
+//   * warp 0 is a TMA producer: per stage of TPR*rounds tiles it issues 1-D bulk
 //     copies (cp.async.bulk, SASS UBLKCP) of every column's contiguous word
 //     range + the matching block_starts slice into a ring of shared-memory
 //     stages, completion tracked by mbarrier transaction counts
@@ -23,8 +23,8 @@ namespace tp {
 
 constexpr int TILE_ROWS = 512;      // D = 4 blocks of 128 = RFOR block
 constexpr int MB_ROWS = 32;         // miniblock
-constexpr int CONSUMER_WARPS = 4;   // 4 warps x 2 tiles = TPS tiles per stage
-constexpr int TPS = 2 * CONSUMER_WARPS;
+constexpr int CONSUMER_WARPS = 4;   // 4 warps x 2 tiles = TPR tiles per consumer round
+constexpr int TPR = 2 * CONSUMER_WARPS;
 constexpr int THREADS = 32 * (CONSUMER_WARPS + 1);
 constexpr int MAX_STREAMS = 2 * 6;  // up to 6 columns, 2 streams each (RFOR)
 constexpr unsigned FULL = 0xffffffffu;
@@ -56,6 +56,21 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
       "@!P1 bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
       "r"(parity)
       : "memory");
+}
+// producer-side wait: the thread may be suspended up to ~0.5 us between probes
+// instead of spinning on the issue slots the consumers need
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, %2;\n\t"
+      "@!P1 bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+      "r"(parity), "r"(500u)
+      : "memory");
+}
+__device__ __forceinline__ void st_shared_v4(uint32_t* p, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
+  asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(smem_u32(p)), "r"(a), "r"(b), "r"(c), "r"(d)
+               : "memory");
 }
 // 1-D bulk copy global -> shared, completes `bytes` on the mbarrier (TMA, UBLKCP)
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar,
@@ -114,6 +129,7 @@ struct Params {
   uint32_t scratch_off; // word offset of per-warp scratch (after the ring)
   uint32_t scratch_words_per_warp;
   uint32_t staging_off; // word offset of the decode->global staging buffers inside a warp's scratch
+  uint32_t rounds;      // consumer rounds per stage: a stage holds TPR * rounds tiles
 };
 
 // ------------------------------------------------------------------ bit unpack
@@ -160,20 +176,25 @@ __device__ __forceinline__ void unpack_any(const uint32_t* __restrict__ w, uint3
   case B:          \
     unpack_fixed<B>(w, e); break;
 
-// Warp-cooperative dispatch: lanes agreeing on b take the specialised path.
+// Warp-cooperative dispatch: the warp runs the specialised routine once per
+// distinct bitwidth among its lanes (one pass when the column's miniblocks share b,
+// the common case; a few passes for sorted-delta or run-length streams).
 __device__ __forceinline__ void unpack_mb(const uint32_t* __restrict__ w, uint32_t b, uint32_t (&e)[32]) {
-  const uint32_t bmin = __reduce_min_sync(FULL, b), bmax = __reduce_max_sync(FULL, b);
-  if (bmin == bmax) {
-    switch (bmin) {
-      TP_CASE(0) TP_CASE(1) TP_CASE(2) TP_CASE(3) TP_CASE(4) TP_CASE(5) TP_CASE(6) TP_CASE(7)
-      TP_CASE(8) TP_CASE(9) TP_CASE(10) TP_CASE(11) TP_CASE(12) TP_CASE(13) TP_CASE(14) TP_CASE(15)
-      TP_CASE(16) TP_CASE(17) TP_CASE(18) TP_CASE(19) TP_CASE(20) TP_CASE(21) TP_CASE(22) TP_CASE(23)
-      TP_CASE(24) TP_CASE(25) TP_CASE(26) TP_CASE(27) TP_CASE(28) TP_CASE(29) TP_CASE(30) TP_CASE(31)
-      default: unpack_fixed<32>(w, e); break;
+  uint32_t todo = FULL;
+  do {
+    const uint32_t bl = __shfl_sync(FULL, b, __ffs(todo) - 1);
+    const bool mine = b == bl;
+    todo &= ~__ballot_sync(FULL, mine);
+    if (mine) {
+      switch (bl) {
+        TP_CASE(0) TP_CASE(1) TP_CASE(2) TP_CASE(3) TP_CASE(4) TP_CASE(5) TP_CASE(6) TP_CASE(7)
+        TP_CASE(8) TP_CASE(9) TP_CASE(10) TP_CASE(11) TP_CASE(12) TP_CASE(13) TP_CASE(14) TP_CASE(15)
+        TP_CASE(16) TP_CASE(17) TP_CASE(18) TP_CASE(19) TP_CASE(20) TP_CASE(21) TP_CASE(22) TP_CASE(23)
+        TP_CASE(24) TP_CASE(25) TP_CASE(26) TP_CASE(27) TP_CASE(28) TP_CASE(29) TP_CASE(30) TP_CASE(31)
+        default: unpack_fixed<32>(w, e); break;
+      }
     }
-  } else {
-    unpack_any(w, b, e);
-  }
+  } while (todo);
 }
 #undef TP_CASE
 
@@ -200,25 +221,26 @@ __device__ __forceinline__ uint64_t sum_fixed(const uint32_t* __restrict__ w) {
 
 #define TP_SCASE(B) \
   case B:           \
-    return sum_fixed<B>(w);
+    r = sum_fixed<B>(w); break;
 
 __device__ __forceinline__ uint64_t sum_mb(const uint32_t* __restrict__ w, uint32_t b) {
-  const uint32_t bmin = __reduce_min_sync(FULL, b), bmax = __reduce_max_sync(FULL, b);
-  if (bmin == bmax) {
-    switch (bmin) {
-      TP_SCASE(0) TP_SCASE(1) TP_SCASE(2) TP_SCASE(3) TP_SCASE(4) TP_SCASE(5) TP_SCASE(6) TP_SCASE(7)
-      TP_SCASE(8) TP_SCASE(9) TP_SCASE(10) TP_SCASE(11) TP_SCASE(12) TP_SCASE(13) TP_SCASE(14) TP_SCASE(15)
-      TP_SCASE(16) TP_SCASE(17) TP_SCASE(18) TP_SCASE(19) TP_SCASE(20) TP_SCASE(21) TP_SCASE(22) TP_SCASE(23)
-      TP_SCASE(24) TP_SCASE(25) TP_SCASE(26) TP_SCASE(27) TP_SCASE(28) TP_SCASE(29) TP_SCASE(30) TP_SCASE(31)
-      default: return sum_fixed<32>(w);
+  uint64_t r = 0;
+  uint32_t todo = FULL;
+  do {
+    const uint32_t bl = __shfl_sync(FULL, b, __ffs(todo) - 1);
+    const bool mine = b == bl;
+    todo &= ~__ballot_sync(FULL, mine);
+    if (mine) {
+      switch (bl) {
+        TP_SCASE(0) TP_SCASE(1) TP_SCASE(2) TP_SCASE(3) TP_SCASE(4) TP_SCASE(5) TP_SCASE(6) TP_SCASE(7)
+        TP_SCASE(8) TP_SCASE(9) TP_SCASE(10) TP_SCASE(11) TP_SCASE(12) TP_SCASE(13) TP_SCASE(14) TP_SCASE(15)
+        TP_SCASE(16) TP_SCASE(17) TP_SCASE(18) TP_SCASE(19) TP_SCASE(20) TP_SCASE(21) TP_SCASE(22) TP_SCASE(23)
+        TP_SCASE(24) TP_SCASE(25) TP_SCASE(26) TP_SCASE(27) TP_SCASE(28) TP_SCASE(29) TP_SCASE(30) TP_SCASE(31)
+        default: r = sum_fixed<32>(w); break;
+      }
     }
-  }
-  uint32_t e[32];
-  unpack_any(w, b, e);
-  uint64_t s = 0;
-#pragma unroll
-  for (int i = 0; i < 32; ++i) s += e[i];
-  return s;
+  } while (todo);
+  return r;
 }
 #undef TP_SCASE
 

@@ -20,10 +20,16 @@ namespace tp {
 std::atomic<uint64_t> g_launches{0};
 
 // ------------------------------------------------------------------ stage context
+// A stage holds TPR * rounds consecutive tiles; consumers walk it in rounds of
+// TPR tiles (each consumer warp: 2 tiles = 32 miniblocks per round).
+constexpr uint32_t VIEW_WORDS = 4 * MAX_STREAMS;  // per-warp table: {lo, dshift, sshift, -} per stream
+
 struct StageCtx {
   const uint32_t* stage;  // this stage's shared words
-  uint32_t tile_base;     // first tile of the stage
-  uint32_t tile_end;      // one past the last tile of the stage (CTA range)
+  const uint32_t* views;  // the warp's per-stage stream table (see stage_views)
+  uint32_t t0s;           // first tile of the stage (global index)
+  uint32_t round_base;    // stage-local index of the round's first tile
+  uint32_t tile_end;      // one past the last tile of the CTA range
 };
 
 struct StreamView {
@@ -33,22 +39,36 @@ struct StreamView {
   uint32_t dshift, sshift;
 };
 
+// Computed once per stage by lane q for stream q (the stage's first copied word and
+// the 16-byte alignment shifts of the two bulk copies), read back by every decode.
+__device__ __forceinline__ void stage_views(const Params& P, uint32_t* views, const uint32_t* stage, uint32_t t0s,
+                                            uint32_t lane) {
+  if (lane < P.nstreams) {
+    const Stream& st = P.st[lane];
+    const uint32_t sidx = st.kind == K_RFOR ? t0s : 4u * t0s;
+    const uint32_t sshift = align_shift(st.starts, sidx);
+    const uint32_t lo = stage[st.starts_off + sshift] - (st.kind == K_DFOR ? 1u : 0u);
+    *reinterpret_cast<uint4*>(views + 4 * lane) = make_uint4(lo, align_shift(st.data, lo), sshift, 0u);
+  }
+  __syncwarp();
+}
+
 __device__ __forceinline__ StreamView stream_view(const Params& P, uint32_t s, const StageCtx& C) {
   const Stream& st = P.st[s];
+  const uint4 t = *reinterpret_cast<const uint4*>(C.views + 4 * s);
   StreamView v;
-  const uint32_t sidx = st.kind == K_RFOR ? C.tile_base : 4u * C.tile_base;
   v.ss = C.stage + st.starts_off;
-  v.sshift = align_shift(st.starts, sidx);
-  v.lo = v.ss[v.sshift] - (st.kind == K_DFOR ? 1u : 0u);
   v.sd = C.stage + st.data_off;
-  v.dshift = align_shift(st.data, v.lo);
+  v.lo = t.x;
+  v.dshift = t.y;
+  v.sshift = t.z;
   return v;
 }
 
-// lane geometry inside a consumer warp: 2 tiles x 16 miniblocks
+// lane geometry inside a consumer warp: 2 tiles x 16 miniblocks per round
 struct Lane {
   uint32_t lane, cw;          // lane id, consumer warp id
-  uint32_t tile_local;        // tile inside the stage
+  uint32_t tile_local;        // tile inside the round (0..TPR-1)
   uint32_t mb;                // miniblock inside the tile (0..15)
 };
 __device__ __forceinline__ Lane lane_geom() {
@@ -60,15 +80,24 @@ __device__ __forceinline__ Lane lane_geom() {
   return g;
 }
 
+// the thread's miniblock of a FOR / DFOR column in this round
+__device__ __forceinline__ MbView for_mb(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
+                                         const StreamView& v, uint32_t& tl, bool& tv) {
+  tl = C.round_base + g.tile_local;  // stage-local tile
+  tv = C.t0s + tl < C.tile_end;
+  const uint32_t lb = 4u * tl + (g.mb >> 2);
+  return for_view(v.sd, v.ss, v.lo, v.dshift, v.sshift, tv ? 4u * C.t0s + lb : UINT_MAX, c.nblocks, lb,
+                  g.mb & 3u);
+}
+
 // ---------------------------------------------------------------- GPU-FOR decode
 // LoadBitPack analogue: the thread's 32 rows of the tile.
 __device__ __forceinline__ void decode_for(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                            uint32_t (&val)[32]) {
   const StreamView v = stream_view(P, c.s0, C);
-  const uint32_t lb = 4u * g.tile_local + (g.mb >> 2);
-  const bool tv = C.tile_base + g.tile_local < C.tile_end;
-  const MbView m = for_view(v.sd, v.ss, v.lo, v.dshift, v.sshift, tv ? 4u * C.tile_base + lb : UINT_MAX,
-                            c.nblocks, lb, g.mb & 3u);
+  uint32_t tl;
+  bool tv;
+  const MbView m = for_mb(P, c, C, g, v, tl, tv);
   uint32_t e[32];
   unpack_mb(m.w, m.b, e);
 #pragma unroll
@@ -83,12 +112,11 @@ __device__ __forceinline__ void decode_for(const Params& P, const Col& c, const 
 __device__ __forceinline__ void decode_dfor(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                             uint32_t (&val)[32]) {
   const StreamView v = stream_view(P, c.s0, C);
-  const uint32_t lb = 4u * g.tile_local + (g.mb >> 2);
-  const bool tv = C.tile_base + g.tile_local < C.tile_end;
-  const MbView m = for_view(v.sd, v.ss, v.lo, v.dshift, v.sshift, tv ? 4u * C.tile_base + lb : UINT_MAX,
-                            c.nblocks, lb, g.mb & 3u);
+  uint32_t tl;
+  bool tv;
+  const MbView m = for_mb(P, c, C, g, v, tl, tv);
   uint32_t first = 0u;
-  if (tv) first = v.sd[v.ss[v.sshift + 4u * g.tile_local] - 1u - v.lo + v.dshift];
+  if (tv) first = v.sd[v.ss[v.sshift + 4u * tl] - 1u - v.lo + v.dshift];
   uint32_t e[32];
   unpack_mb(m.w, m.b, e);
   uint32_t run = 0u;
@@ -104,108 +132,112 @@ __device__ __forceinline__ void decode_dfor(const Params& P, const Col& c, const
 }
 
 // ---------------------------------------------------------------- GPU-RFOR decode
-// LoadRBitPack analogue: unpack the value and run-length stream
-// blocks of the row block (lane j of a 16-lane half takes entries 32j..32j+31
-// of both streams), exclusive scan of the run lengths -> run starts S, then
-// each thread expands its 32 rows by a search + forward walk over S in the
-// warp's scratch (result == repeat(V, L), R19).
-__device__ __forceinline__ uint32_t pad33(uint32_t e) { return e + (e >> 5); }
-constexpr uint32_t RFOR_HALF_WORDS = 1072;  // S (529) + V (528), padded so the halves' banks differ by 16
+// LoadRBitPack analogue.  Per row block (a warp does 2 per round):
+//  1. lane-per-entry unpack of the value and run-length stream blocks, 32 entries
+//     (= one miniblock, warp-uniform bitwidth) per step;
+//  2. warp scan of the run lengths -> run start rows S (the first inclusive scan of [18]);
+//  3. scatter: value V_e -> smem, bit S_e -> a 512-bit run-start bitmap (the scatters of [18]);
+//  4. expand: the thread owning rows 32j..32j+31 counts run starts before its rows
+//     (popcount + 16-lane scan = the second scan of [18]) and walks its bitmap word.
+// The result equals repeat(V, L) (R19).
+constexpr uint32_t RFOR_HALF_WORDS = 16 + 512 + 32;  // bitmap + values + pad: the halves sit 16 banks apart
 constexpr uint32_t RFOR_SCRATCH_WORDS = 2 * RFOR_HALF_WORDS;
 
-struct RforHdr {
-  const uint32_t* w;
-  uint32_t ref, b, r, cnt;
-};
-__device__ __forceinline__ RforHdr rfor_hdr(const StreamView& v, uint32_t tile_local, uint32_t j, bool tv) {
-  RforHdr h;
-  h.r = 0u; h.cnt = 0u; h.ref = 0u; h.b = 0u; h.w = v.sd;
-  if (!tv) return h;
-  const uint32_t* blk = v.sd + (v.ss[v.sshift + tile_local] - v.lo + v.dshift);
-  h.r = blk[0];       // run / value count
-  h.ref = blk[1];
-  uint32_t off = 0u;
+__device__ __forceinline__ uint32_t warp_inclusive_scan(uint32_t x, uint32_t lane) {
 #pragma unroll
-  for (uint32_t q = 0; q < 4; ++q) {
-    const uint32_t bw = blk[2 + q];
-    if (q < (j >> 2)) off += (bw * 0x01010101u) >> 24;
-    else if (q == (j >> 2)) { off += bw_prefix(bw, j & 3u); h.b = min((bw >> (8u * (j & 3u))) & 255u, 32u); }
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t y = __shfl_up_sync(FULL, x, d);
+    if (lane >= (uint32_t)d) x += y;
   }
-  h.w = blk + 6u + off;  // [r][ref][4 bitwidth words] then tight miniblocks (R17)
-  const int rem = (int)h.r - 32 * (int)j;
-  h.cnt = rem <= 0 ? 0u : (rem >= 32 ? 32u : (uint32_t)rem);
-  return h;
+  return x;
+}
+
+// entry `lane` of a b-bit miniblock at m (lane-per-entry); `mask` = 2^b - 1
+__device__ __forceinline__ uint32_t extract_lane(const uint32_t* m, uint32_t lane, uint32_t b, uint32_t mask) {
+  const uint32_t p = lane * b;
+  const uint32_t* w = m + (p >> 5);
+  return __funnelshift_r(w[0], w[1], p) & mask;  // the funnel shift uses p mod 32
 }
 
 __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                             uint32_t* scratch, uint32_t (&val)[32]) {
   const StreamView vv = stream_view(P, c.s0, C), vl = stream_view(P, c.s1, C);
-  const bool tv = C.tile_base + g.tile_local < C.tile_end;
-  const uint32_t j = g.mb;
-  const RforHdr hv = rfor_hdr(vv, g.tile_local, j, tv), hl = rfor_hdr(vl, g.tile_local, j, tv);  // hv.r == hl.r
-  uint32_t* S = scratch + (g.lane >> 4) * RFOR_HALF_WORDS;
-  uint32_t* V = S + 529;
-  uint32_t ev[32], el[32];
-  unpack_mb(hv.w, hv.b, ev);
-  unpack_mb(hl.w, hl.b, el);
-  // local exclusive scan of the run lengths of entries 32j..32j+cnt-1
-  uint32_t run = 0u;
-#pragma unroll
-  for (int i = 0; i < 32; ++i) {
-    const uint32_t len = (uint32_t)i < hl.cnt ? hl.ref + el[i] : 0u;
-    el[i] = run;
-    run += len;
-  }
-  const uint32_t incl = seg16_inclusive_scan(run);
-  const uint32_t sbase = incl - run;
-#pragma unroll
-  for (int i = 0; i < 32; ++i) {
-    if ((uint32_t)i < hl.cnt) {
-      S[33u * j + i] = sbase + el[i];
-      V[33u * j + i] = hv.ref + ev[i];
-    }
-  }
-  if (j == 0 && hl.r > 0u) S[pad33(hl.r)] = 0x7fffffffu;  // sentinel
-  __syncwarp();
-  // expand: rows 32j .. 32j+31 of the row block
-  const uint32_t row0 = 32u * j, r = hl.r;
-  if (r > 0u) {
-    uint32_t a = 0u, bnd = r;
-    while (bnd - a > 1u) {
-      const uint32_t mid = (a + bnd) >> 1;
-      if (S[pad33(mid)] <= row0) a = mid; else bnd = mid;
-    }
-    uint32_t cur = a, nxt = S[pad33(a + 1u)], x = V[pad33(a)];
-#pragma unroll
-    for (int i = 0; i < 32; ++i) {
-      if (row0 + i >= nxt) {
-        ++cur;
-        x = V[pad33(cur)];
-        nxt = S[pad33(cur + 1u)];
+  const uint32_t lane = g.lane;
+#pragma unroll 1
+  for (uint32_t h = 0; h < 2; ++h) {
+    uint32_t* bitmap = scratch + h * RFOR_HALF_WORDS;
+    uint32_t* V = bitmap + 16;
+    const uint32_t tl = C.round_base + 2u * g.cw + h;
+    const bool tv = C.t0s + tl < C.tile_end;
+    if (lane < 16) bitmap[lane] = 0u;
+    __syncwarp();
+    if (!tv) continue;  // warp-uniform
+    const uint32_t* bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
+    const uint32_t* bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
+    const uint32_t r = min(bV[0], 512u);  // run / value count
+    const uint32_t nq = (r + 31u) >> 5;
+    const uint32_t refV = bV[1], refL = bL[1];  // references (FOR on both arrays)
+    const uint8_t* bwV = reinterpret_cast<const uint8_t*>(bV + 2);  // bitwidth byte q = miniblock q (R2, R17)
+    const uint8_t* bwL = reinterpret_cast<const uint8_t*>(bL + 2);
+    const uint32_t* mV = bV + 6;  // [r][ref][4 bitwidth words] then the tight miniblocks (R17)
+    const uint32_t* mL = bL + 6;
+    uint32_t carry = 0u;
+    for (uint32_t q = 0; q < nq; ++q) {  // one miniblock (32 entries) of each stream per step
+      const uint32_t bv = min((uint32_t)bwV[q], 32u), bl = min((uint32_t)bwL[q], 32u);
+      const uint32_t mv = __funnelshift_lc(0xffffffffu, 0u, bv), ml = __funnelshift_lc(0xffffffffu, 0u, bl);
+      const uint32_t e = 32u * q + lane;
+      const bool in = e < r;
+      // 1. lane-per-entry unpack (warp-uniform bitwidth per miniblock)
+      const uint32_t xv = refV + extract_lane(mV, lane, bv, mv);
+      const uint32_t xl = in ? refL + extract_lane(mL, lane, bl, ml) : 0u;
+      // 2. scan of the run lengths -> run start rows
+      const uint32_t incl = warp_inclusive_scan(xl, lane);
+      const uint32_t S = carry + incl - xl;
+      // 3. scatter the value and the run-start bit
+      if (in) {
+        V[e] = xv;
+        atomicOr(&bitmap[(S >> 5) & 15u], 1u << (S & 31u));
       }
-      val[i] = x;
+      carry += __shfl_sync(FULL, incl, 31);
+      mV += bv;  // full miniblocks occupy b words; only the last one can be partial
+      mL += bl;
     }
-  } else {
+  }
+  __syncwarp();
+  // 4. expand: rows 32j .. 32j+31 of row block h
+  const uint32_t h = lane >> 4, j = lane & 15u;
+  const uint32_t* bitmap = scratch + h * RFOR_HALF_WORDS;
+  const uint32_t* V = bitmap + 16;
+  const uint32_t bm = bitmap[j];
+  const uint32_t pc = __popc(bm);
+  const int before = (int)(seg16_inclusive_scan(pc) - pc);  // run starts before row 32j
 #pragma unroll
-    for (int i = 0; i < 32; ++i) val[i] = 0u;
+  for (int i = 0; i < 32; ++i) {
+    const int cur = before - 1 + __popc(bm & (0xffffffffu >> (31 - i)));
+    val[i] = V[cur < 0 ? 0 : cur];
   }
   __syncwarp();
 }
 
+// MASK: which decoders a kernel instantiation carries (bit 1 << scheme); kernels
+// are instantiated per scheme mix so that FOR-only kernels keep FOR's register budget.
+constexpr uint32_t M_FOR = 1u << S_FOR, M_DFOR = 1u << S_DFOR, M_RFOR = 1u << S_RFOR;
+template <uint32_t MASK>
 __device__ __forceinline__ void decode_col(const Params& P, uint32_t ci, const StageCtx& C, const Lane& g,
                                            uint32_t* scratch, uint32_t (&val)[32]) {
   const Col& c = P.col[ci];
-  if (c.scheme == S_FOR) decode_for(P, c, C, g, val);
-  else if (c.scheme == S_DFOR) decode_dfor(P, c, C, g, val);
-  else decode_rfor(P, c, C, g, scratch, val);
+  if ((MASK & M_FOR) && c.scheme == S_FOR) decode_for(P, c, C, g, val);
+  else if ((MASK & M_DFOR) && c.scheme == S_DFOR) decode_dfor(P, c, C, g, val);
+  else if (MASK & M_RFOR) decode_rfor(P, c, C, g, scratch, val);
 }
 
 // ------------------------------------------------------------------ the pipeline
-// warp 0: TMA producer; warps 1..CONSUMER_WARPS: consumers (Op::stage).
+// warp 0: TMA producer; warps 1..CONSUMER_WARPS: consumers (Op::stage per round).
 template <class Op>
 __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
   extern __shared__ __align__(1024) uint32_t smem[];
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
+  const uint32_t TPS = TPR * P.rounds;  // tiles per stage
   // CTA tile range, in pairs of tiles so that a consumer warp's 1024 rows
   // never straddle two CTAs (decode->global stores whole warp boxes)
   const uint32_t npairs = (P.ntiles + 1u) >> 1;
@@ -244,7 +276,7 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
       const uint32_t se = min(sb + 31, nst);
       for (uint32_t s = sb; s < se; ++s) {
         const uint32_t slot = s % P.nstages;
-        if (s >= P.nstages) mbar_wait(&empty[slot], ((s / P.nstages) + 1u) & 1u);
+        if (s >= P.nstages) mbar_wait_sleep(&empty[slot], ((s / P.nstages) + 1u) & 1u);
         const uint32_t tile_base = t0 + s * TPS, tile_end = min(tile_base + TPS, t1);
         uint32_t mylo = 0u, myhi = 0u;
 #pragma unroll
@@ -290,15 +322,23 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
   } else {
     // ---------------- consumers
     const Lane g = lane_geom();
-    uint32_t* scratch = smem + P.scratch_off + g.cw * P.scratch_words_per_warp;
+    uint32_t* views = smem + P.scratch_off + g.cw * P.scratch_words_per_warp;
+    uint32_t* scratch = views + VIEW_WORDS;
+    uint32_t rc = 0;  // round counter (decode->global buffer parity)
     for (uint32_t s = 0; s < nst; ++s) {
       const uint32_t slot = s % P.nstages;
       mbar_wait(&full[slot], (s / P.nstages) & 1u);
       StageCtx C;
       C.stage = smem + slot * P.stage_words;
-      C.tile_base = t0 + s * TPS;
-      C.tile_end = min(C.tile_base + TPS, t1);
-      op.stage(P, C, g, scratch, s);
+      C.views = views;
+      C.t0s = t0 + s * TPS;
+      stage_views(P, views, C.stage, C.t0s, g.lane);
+      C.tile_end = t1;
+      const uint32_t nr = min(P.rounds, (t1 - C.t0s + TPR - 1) / TPR);
+      for (uint32_t r = 0; r < nr; ++r, ++rc) {
+        C.round_base = r * TPR;
+        op.stage(P, C, g, scratch, rc);
+      }
       __syncwarp();
       if (g.lane == 0) mbar_arrive(&empty[slot]);
     }
@@ -314,19 +354,20 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t x) {
 }
 
 // decode -> sum (decode-only microbenchmark)
+template <uint32_t MASK>
 struct SumOp {
   unsigned long long* out;
   uint64_t acc;
   __device__ void stage(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t) {
     const Col& c = P.col[0];
-    const uint32_t tile = C.tile_base + g.tile_local;
+    const uint32_t tile = C.t0s + C.round_base + g.tile_local;
     const uint32_t row0 = tile * TILE_ROWS + g.mb * MB_ROWS;
     const bool tv = tile < C.tile_end;
-    if (c.scheme == S_FOR) {
+    if (MASK == M_FOR) {
       const StreamView v = stream_view(P, c.s0, C);
-      const uint32_t lb = 4u * g.tile_local + (g.mb >> 2);
-      const MbView m = for_view(v.sd, v.ss, v.lo, v.dshift, v.sshift, tv ? 4u * C.tile_base + lb : UINT_MAX,
-                                c.nblocks, lb, g.mb & 3u);
+      uint32_t tl;
+      bool tv2;
+      const MbView m = for_mb(P, c, C, g, v, tl, tv2);
       if (tv && row0 + MB_ROWS <= P.n) {
         const uint64_t se = sum_mb(m.w, m.b);
         acc += se + (uint64_t)((int64_t)(int32_t)m.ref * 32);
@@ -339,7 +380,7 @@ struct SumOp {
       }
     } else {
       uint32_t val[32];
-      decode_col(P, 0, C, g, scratch, val);
+      decode_col<MASK>(P, 0, C, g, scratch, val);
       if (tv && row0 + MB_ROWS <= P.n) {
 #pragma unroll
         for (int i = 0; i < 32; ++i) acc += (uint64_t)(int64_t)(int32_t)val[i];
@@ -359,14 +400,15 @@ struct SumOp {
 // decode -> global (Fig. 7a mode): the warp's 1024 rows go to a
 // 128B-swizzled 4 KB shared buffer (conflict-free 16-byte stores) and leave by
 // one TMA tensor store; the partial last miniblock (n % 32 rows) is stored directly.
+template <uint32_t MASK>
 struct GlobalOp {
   const CUtensorMap* tmap;
   int32_t* out;
   uint32_t full_rows32;  // n / 32: rows of the [n/32][32] tensor
   __device__ void stage(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t s) {
     uint32_t val[32];
-    decode_col(P, 0, C, g, scratch, val);
-    const uint32_t pair_tile = C.tile_base + 2u * g.cw;
+    decode_col<MASK>(P, 0, C, g, scratch, val);
+    const uint32_t pair_tile = C.t0s + C.round_base + 2u * g.cw;
     if (pair_tile >= C.tile_end) return;  // warp-uniform
     // staging buffers: 2 x 4 KB per warp, 1024-aligned, after the RFOR scratch
     uint32_t* buf = scratch + P.staging_off;
@@ -377,8 +419,8 @@ struct GlobalOp {
     const uint32_t l = g.lane;
 #pragma unroll
     for (uint32_t q = 0; q < 8; ++q) {
-      uint4 v4 = make_uint4(val[4 * q], val[4 * q + 1], val[4 * q + 2], val[4 * q + 3]);
-      *reinterpret_cast<uint4*>(buf + l * 32u + ((q ^ (l & 7u)) << 2)) = v4;
+      st_shared_v4(buf + l * 32u + ((q ^ (l & 7u)) << 2), val[4 * q], val[4 * q + 1], val[4 * q + 2],
+                   val[4 * q + 3]);
     }
     fence_proxy_async_smem();
     __syncwarp();
@@ -400,53 +442,67 @@ struct GlobalOp {
   }
 };
 
-// select / project / aggregate over up to 6 columns
+// select / project / aggregate over up to 6 columns.  The host orders
+// the columns predicate-only first, then the projection operands a and b, so that
+// at most two decoded miniblocks are live at a time.
+struct SelectArgs {
+  int32_t lo[TP_MAX_COLS], hi[TP_MAX_COLS];  // per position in `order`
+  uint32_t order[TP_MAX_COLS];               // column index per position
+  uint32_t npred;                            // positions [0, npred) are predicate-only
+  int proj;                                  // TP_PROJ_*
+  uint32_t has_a, has_b;                     // positions npred (a) and npred+1 (b) present
+};
+
+template <uint32_t MASK>
 struct SelectOp {
-  int32_t lo[TP_MAX_COLS], hi[TP_MAX_COLS];
-  int proj, a, b;
+  const SelectArgs* A;
   unsigned long long* out;
   uint64_t acc;
+  __device__ __forceinline__ void pred(uint32_t k, const uint32_t (&v)[32], uint32_t& alive) const {
+    const int32_t l = A->lo[k], h = A->hi[k];
+#pragma unroll
+    for (int i = 0; i < 32; ++i) {
+      const int32_t x = (int32_t)v[i];
+      if (x < l || x > h) alive &= ~(1u << i);
+    }
+  }
   __device__ void stage(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t) {
-    const uint32_t tile = C.tile_base + g.tile_local;
+    const uint32_t tile = C.t0s + C.round_base + g.tile_local;
     const uint32_t row0 = tile * TILE_ROWS + g.mb * MB_ROWS;
     uint32_t alive = 0u;
     if (tile < C.tile_end && row0 < P.n) {
       const uint32_t nrows = P.n - row0;
       alive = nrows >= 32u ? 0xffffffffu : ((1u << nrows) - 1u);
     }
-    uint32_t va[32], vb[32];
-#pragma unroll
-    for (int i = 0; i < 32; ++i) { va[i] = 0u; vb[i] = 0u; }
-    for (uint32_t c = 0; c < P.ncols; ++c) {
+    const uint32_t nk = A->npred + A->has_a + A->has_b;
+    const uint32_t ka = A->has_a ? A->npred : 0xffffffffu;
+    const uint32_t kb = A->has_b ? A->npred + 1u : 0xffffffffu;
+    const bool mul = A->proj == TP_PROJ_MUL;
+    uint32_t va[32];
+    for (uint32_t k = 0; k < nk; ++k) {  // one decode call site: keeps the kernel small
       uint32_t v[32];
-      decode_col(P, c, C, g, scratch, v);
-      const int32_t l = lo[c], h = hi[c];
+      decode_col<MASK>(P, A->order[k], C, g, scratch, v);
+      pred(k, v, alive);
+      if (k == ka) {
+        if (A->has_b) {
 #pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        const int32_t x = (int32_t)v[i];
-        if (x < l || x > h) alive &= ~(1u << i);
-      }
-      if ((int)c == a) {
+          for (int i = 0; i < 32; ++i) va[i] = v[i];
+        } else {
 #pragma unroll
-        for (int i = 0; i < 32; ++i) va[i] = v[i];
-      }
-      if ((int)c == b) {
+          for (int i = 0; i < 32; ++i)
+            if (alive & (1u << i)) acc += (uint64_t)(int64_t)(int32_t)v[i];
+        }
+      } else if (k == kb) {
 #pragma unroll
-        for (int i = 0; i < 32; ++i) vb[i] = v[i];
-      }
-    }
-#pragma unroll
-    for (int i = 0; i < 32; ++i) {
-      if (alive & (1u << i)) {
-        int64_t t;
-        const int64_t xa = (int32_t)va[i], xb = (int32_t)vb[i];
-        if (proj == TP_PROJ_COL) t = xa;
-        else if (proj == TP_PROJ_MUL) t = xa * xb;
-        else if (proj == TP_PROJ_SUB) t = xa - xb;
-        else t = 1;
-        acc += (uint64_t)t;
+        for (int i = 0; i < 32; ++i) {
+          if (alive & (1u << i)) {
+            const int64_t xa = (int32_t)va[i], xb = (int32_t)v[i];
+            acc += (uint64_t)(mul ? xa * xb : xa - xb);
+          }
+        }
       }
     }
+    if (A->proj == TP_PROJ_COUNT) acc += __popc(alive);
   }
   __device__ void finish(const Params&, const Lane& g) {
     const uint64_t s = warp_sum_u64(acc);
@@ -454,31 +510,29 @@ struct SelectOp {
   }
 };
 
-__global__ void __launch_bounds__(THREADS) k_decode_sum(const __grid_constant__ Params P, unsigned long long* out) {
-  SumOp op;
+template <uint32_t MASK>
+__global__ void __launch_bounds__(THREADS, 4) k_decode_sum(const __grid_constant__ Params P, unsigned long long* out) {
+  SumOp<MASK> op;
   op.out = out;
   op.acc = 0;
   run_pipeline(P, op);
 }
 
-__global__ void __launch_bounds__(THREADS)
+template <uint32_t MASK>
+__global__ void __launch_bounds__(THREADS, 4)
     k_decode_global(const __grid_constant__ Params P, const __grid_constant__ CUtensorMap tmap, int32_t* out) {
-  GlobalOp op;
+  GlobalOp<MASK> op;
   op.tmap = &tmap;
   op.out = out;
   op.full_rows32 = P.n >> 5;
   run_pipeline(P, op);
 }
 
-struct SelectArgs {
-  int32_t lo[TP_MAX_COLS], hi[TP_MAX_COLS];
-  int proj, a, b;
-};
-__global__ void __launch_bounds__(THREADS)
+template <uint32_t MASK>
+__global__ void __launch_bounds__(THREADS, 2)
     k_select_sum(const __grid_constant__ Params P, const __grid_constant__ SelectArgs A, unsigned long long* out) {
-  SelectOp op;
-  for (int c = 0; c < TP_MAX_COLS; ++c) { op.lo[c] = A.lo[c]; op.hi[c] = A.hi[c]; }
-  op.proj = A.proj; op.a = A.a; op.b = A.b;
+  SelectOp<MASK> op;
+  op.A = &A;
   op.out = out;
   op.acc = 0;
   run_pipeline(P, op);
@@ -527,8 +581,9 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
   if (!cols || ncols < 1 || ncols > TP_MAX_COLS) return TP_EINVAL;
   const uint64_t n = cols[0].n;
   if (n >= (1ull << 32)) return TP_EUNSUPPORTED;
-  uint32_t off = 0;
   bool any_rfor = false;
+  uint32_t mtws[MAX_STREAMS];
+  uint32_t round_words = 0;  // data words of one round (TPR tiles) over all streams, upper bound
   for (int c = 0; c < ncols; ++c) {
     const tp_column& k = cols[c];
     if (k.n != n) return TP_EINVAL;
@@ -555,25 +610,36 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
       st.nblocks = (uint32_t)k.num_blocks;
       uint32_t mtw = s == 0 ? k.max_tile_words0 : k.max_tile_words1;
       if (mtw == 0 || mtw > worst_tile_words(k.scheme)) mtw = worst_tile_words(k.scheme);
-      st.data_off = off;
-      off += align4(std::max<uint32_t>(TPS * mtw + 12u, 48u));
-      st.starts_off = off;
-      off += align4((rf ? TPS + 1u : 4u * TPS + 1u) + 8u);
+      mtws[P.nstreams] = mtw;
+      round_words += TPR * mtw;
       if (s == 0) cc.s0 = P.nstreams; else cc.s1 = P.nstreams;
       ++P.nstreams;
     }
+  }
+  // rounds per stage: a stage carries ~16 KB of compressed words (bytes in flight for
+  // low bitwidths, where a round of 8 tiles is only a few hundred bytes), at most 8 rounds
+  const uint32_t target_words = 4096;
+  P.rounds = std::max<uint32_t>(1u, std::min<uint32_t>(8u, target_words / std::max<uint32_t>(round_words, 1u)));
+  const uint32_t TPS = TPR * P.rounds;
+  uint32_t off = 0;
+  for (uint32_t q = 0; q < P.nstreams; ++q) {
+    Stream& st = P.st[q];
+    st.data_off = off;
+    off += align4(std::max<uint32_t>(TPS * mtws[q] + 12u, 48u));  // + alignment slop + unpack over-read
+    st.starts_off = off;
+    off += align4((st.kind == K_RFOR ? TPS + 1u : 4u * TPS + 1u) + 8u);
   }
   P.ncols = (uint32_t)ncols;
   P.n = (uint32_t)n;
   P.ntiles = (uint32_t)((n + TILE_ROWS - 1) / TILE_ROWS);
   P.stage_words = align4(off);
-  P.staging_off = any_rfor ? RFOR_SCRATCH_WORDS : 0u;
-  const uint32_t scratch = P.staging_off + extra_scratch;
+  P.staging_off = any_rfor ? RFOR_SCRATCH_WORDS : 0u;  // relative to the scratch after the view table
+  const uint32_t scratch = VIEW_WORDS + P.staging_off + extra_scratch;
   P.scratch_words_per_warp = align4(scratch);
-  // ring depth: up to 4 stages, keep the CTA under ~100 KB so >= 2 CTAs fit an SM
-  uint32_t nstg = 4;
-  while (nstg > 2 && (size_t)(nstg * P.stage_words + CONSUMER_WARPS * P.scratch_words_per_warp) * 4 > 100 * 1024)
-    --nstg;
+  // ring depth: 2..6 stages within ~40 KB so that 4+ CTAs (16+ consumer warps) fit an SM;
+  // 4 CTAs x 40 KB keeps ~100+ KB of TMA traffic in flight per SM
+  uint32_t nstg = 6;
+  while (nstg > 2 && (size_t)nstg * P.stage_words * 4 > 40 * 1024) --nstg;
   P.nstages = nstg;
   P.scratch_off = nstg * P.stage_words;
   smem_bytes = (size_t)(P.scratch_off + CONSUMER_WARPS * P.scratch_words_per_warp) * 4 + 2 * nstg * 8 + 16;
@@ -588,6 +654,18 @@ static int grid_for(K kernel, size_t smem) {
   if (occ < 1) occ = 1;
   if (occ > 8) occ = 8;
   return sm_count() * occ;
+}
+
+static uint32_t scheme_mask(const Params& P) {
+  uint32_t m = 0;
+  for (uint32_t c = 0; c < P.ncols; ++c) m |= 1u << P.col[c].scheme;
+  return m;
+}
+
+template <class K, class... Args>
+static void launch(K kernel, size_t smem, int cap, void* stream, Args... args) {
+  const int grid = std::max(1, std::min<int>(grid_for(kernel, smem), cap));
+  kernel<<<grid, THREADS, smem, (cudaStream_t)stream>>>(args...);
 }
 
 static tp_status launched() {
@@ -620,8 +698,13 @@ tp_status tp_decode_sum(const tp_column* dcol, int64_t* d_sum, void* stream) {
   size_t smem = 0;
   tp_status st = build_params(dcol, 1, 0, P, smem);
   if (st != TP_OK) return st;
-  const int grid = std::min<int>(grid_for(k_decode_sum, smem), (int)((P.ntiles + 1) / 2));
-  k_decode_sum<<<grid, THREADS, smem, (cudaStream_t)stream>>>(P, reinterpret_cast<unsigned long long*>(d_sum));
+  auto out = reinterpret_cast<unsigned long long*>(d_sum);
+  const int cap = (int)((P.ntiles + 1) / 2);
+  switch (scheme_mask(P)) {
+    case M_FOR: launch(k_decode_sum<M_FOR>, smem, cap, stream, P, out); break;
+    case M_DFOR: launch(k_decode_sum<M_DFOR>, smem, cap, stream, P, out); break;
+    default: launch(k_decode_sum<M_RFOR>, smem, cap, stream, P, out); break;
+  }
   return launched();
 }
 
@@ -649,8 +732,12 @@ tp_status tp_decode(const tp_column* dcol, int32_t* d_out, void* stream) {
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return TP_ECUDA;
   }
-  const int grid = std::min<int>(grid_for(k_decode_global, smem), (int)((P.ntiles + 1) / 2));
-  k_decode_global<<<grid, THREADS, smem, (cudaStream_t)stream>>>(P, tmap, d_out);
+  const int cap = (int)((P.ntiles + 1) / 2);
+  switch (scheme_mask(P)) {
+    case M_FOR: launch(k_decode_global<M_FOR>, smem, cap, stream, P, tmap, d_out); break;
+    case M_DFOR: launch(k_decode_global<M_DFOR>, smem, cap, stream, P, tmap, d_out); break;
+    default: launch(k_decode_global<M_RFOR>, smem, cap, stream, P, tmap, d_out); break;
+  }
   return launched();
 }
 
@@ -667,13 +754,30 @@ tp_status tp_select_project_sum(const tp_column* dcols, int ncols, const int32_t
   if (st != TP_OK) return st;
   SelectArgs A;
   memset(&A, 0, sizeof(A));
-  for (int c = 0; c < TP_MAX_COLS; ++c) {
-    A.lo[c] = c < ncols ? lo[c] : INT_MIN;
-    A.hi[c] = c < ncols ? hi[c] : INT_MAX;
+  A.proj = proj_op;
+  const bool use_a = proj_op != TP_PROJ_COUNT, use_b = proj_op == TP_PROJ_MUL || proj_op == TP_PROJ_SUB;
+  uint32_t k = 0;
+  for (int c = 0; c < ncols; ++c) {  // predicate-only columns first
+    if ((use_a && c == a) || (use_b && c == b)) continue;
+    A.order[k] = (uint32_t)c; A.lo[k] = lo[c]; A.hi[k] = hi[c]; ++k;
   }
-  A.proj = proj_op; A.a = a; A.b = b;
-  const int grid = std::min<int>(grid_for(k_select_sum, smem), (int)((P.ntiles + 1) / 2));
-  k_select_sum<<<grid, THREADS, smem, (cudaStream_t)stream>>>(P, A, reinterpret_cast<unsigned long long*>(d_result));
+  A.npred = k;
+  if (use_a) { A.order[k] = (uint32_t)a; A.lo[k] = lo[a]; A.hi[k] = hi[a]; ++k; A.has_a = 1; }
+  if (use_b) {
+    // a == b (e.g. sum of squares) decodes the column twice; predicates are idempotent
+    A.order[k] = (uint32_t)b; A.lo[k] = lo[b]; A.hi[k] = hi[b]; ++k; A.has_b = 1;
+  }
+  auto out = reinterpret_cast<unsigned long long*>(d_result);
+  const int cap = (int)((P.ntiles + 1) / 2);
+  switch (scheme_mask(P)) {
+    case M_FOR: launch(k_select_sum<M_FOR>, smem, cap, stream, P, A, out); break;
+    case M_DFOR: launch(k_select_sum<M_DFOR>, smem, cap, stream, P, A, out); break;
+    case M_RFOR: launch(k_select_sum<M_RFOR>, smem, cap, stream, P, A, out); break;
+    case M_FOR | M_DFOR: launch(k_select_sum<M_FOR | M_DFOR>, smem, cap, stream, P, A, out); break;
+    case M_FOR | M_RFOR: launch(k_select_sum<M_FOR | M_RFOR>, smem, cap, stream, P, A, out); break;
+    case M_DFOR | M_RFOR: launch(k_select_sum<M_DFOR | M_RFOR>, smem, cap, stream, P, A, out); break;
+    default: launch(k_select_sum<M_FOR | M_DFOR | M_RFOR>, smem, cap, stream, P, A, out); break;
+  }
   return launched();
 }
 
@@ -699,7 +803,7 @@ tp_status tp_device_info(int* sms, int* ctas_per_sm) {
     Params P;
     size_t smem = 0;
     build_params(&c, 1, 0, P, smem);
-    *ctas_per_sm = grid_for(k_decode_sum, smem) / sm_count();
+    *ctas_per_sm = grid_for(k_decode_sum<M_FOR>, smem) / sm_count();
   }
   return TP_OK;
 }
