@@ -368,7 +368,7 @@ def run_sweep(args, tp, dev, stream, torch):
         flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
         ts = []
         for _ in range(10):
-            flush.zero_()  # L2 flush (small columns fit L2)
+            flush.sum()  # L2 flush by reading (no dirty lines to write back)
             a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record(stream)
             tp.tp_decode_sum(d.col, acc, stream)

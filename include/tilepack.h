@@ -149,6 +149,54 @@ tp_status tp_select_project_sum(const tp_column* dcols, int ncols,
                                 int proj_op, int a, int b,
                                 int64_t* d_result, void* stream);
 
+/* ---------------------------------------------------- star-join queries
+ * The SSB workload of P:1874-1888 (13 queries, dictionary-encoded):
+ * decoded fact-table foreign keys probe dimension lookup tables (Crystal-style
+ * perfect hashing: table[key - key_min]), payloads form a dense group index,
+ * and the measures are aggregated per group -- all inside one tile kernel
+ * (SURVEY 8(a) rows a7-a8).
+ *
+ * tp_lookup_build: DEVICE table[0..table_len) := -1, then for every dimension
+ * row i whose attributes pass all preds:
+ *     table[keys[i] - key_min] = payload ? payload[i] : 0
+ * pred p passes when lo1 <= attr[i] <= hi1 OR lo2 <= attr[i] <= hi2
+ * (set lo2 > hi2 for a single range).  keys/attr/payload are DEVICE int32
+ * arrays of nrows; keys must lie in [key_min, key_min + table_len); payloads
+ * must be >= 0.  npreds <= 4.  Two kernels, asynchronous on `stream`. */
+typedef struct {
+  const int32_t* attr;
+  int32_t lo1, hi1, lo2, hi2;
+} tp_dim_pred;
+tp_status tp_lookup_build(const int32_t* d_keys, uint64_t nrows, int32_t key_min, uint32_t table_len,
+                          const tp_dim_pred* preds, int npreds, const int32_t* d_payload,
+                          int32_t* d_table, void* stream);
+
+/* tp_star_query: one fused pass over ncols (<= TP_MAX_COLS) DEVICE columns
+ * of equal n.  roles[c] says what column c does, applied in the order given:
+ *   TP_ROLE_RANGE   : row survives iff lo <= v <= hi
+ *   TP_ROLE_PROBE   : p = table[v - key_min] (v outside the table -> -1);
+ *                     row survives iff p >= 0; group += p * stride
+ *   TP_ROLE_MEASURE : the row's measure (lo/hi also filter it: use
+ *                     [INT32_MIN, INT32_MAX] for none); agg (below) combines
+ *                     the measures: TP_AGG_SUM: sum(m0); TP_AGG_MUL:
+ *                     sum(m0 * m1); TP_AGG_SUB: sum(m0 - m1)  (int64, R24)
+ * Put MEASURE columns last; with TP_AGG_SUB only m0 may carry a filter.  For every surviving row:
+ *   d_sums[group] += aggregate, d_counts[group] += 1
+ * (DEVICE int64 / uint64 arrays of ngroups, caller-zeroed).  Rows whose group
+ * is >= ngroups are a caller error (not checked per row). */
+enum { TP_ROLE_RANGE = 0, TP_ROLE_PROBE = 1, TP_ROLE_MEASURE = 2 };
+enum { TP_AGG_SUM = 0, TP_AGG_MUL = 1, TP_AGG_SUB = 2 };
+typedef struct {
+  int32_t role;
+  int32_t lo, hi;            /* RANGE */
+  const int32_t* table;      /* PROBE (DEVICE) */
+  int32_t key_min;
+  uint32_t table_len;
+  uint32_t stride;
+} tp_star_col;
+tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int ncols, int agg,
+                        int64_t* d_sums, uint64_t* d_counts, uint32_t ngroups, void* stream);
+
 /* The uncompressed baseline "None": *d_sum += sum of the n int32
  * values of DEVICE array d_x (16-byte aligned), 128-bit streaming loads.
  * Used as the measured HBM read roof of the same consumer. */

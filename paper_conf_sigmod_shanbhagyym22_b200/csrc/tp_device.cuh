@@ -129,7 +129,9 @@ struct Params {
   uint32_t scratch_off; // word offset of per-warp scratch (after the ring)
   uint32_t scratch_words_per_warp;
   uint32_t staging_off; // word offset of the decode->global staging buffers inside a warp's scratch
-  uint32_t rounds;      // consumer rounds per stage: a stage holds TPR * rounds tiles
+  uint32_t rounds;      // consumer rounds per item: an item holds TPR * rounds tiles of one column
+  uint32_t agg_off;     // word offset of the per-CTA aggregation table
+  uint32_t bar_off;     // word offset of the mbarriers (8-byte aligned)
 };
 
 // ------------------------------------------------------------------ bit unpack
@@ -223,8 +225,24 @@ __device__ __forceinline__ uint64_t sum_fixed(const uint32_t* __restrict__ w) {
   case B:           \
     r = sum_fixed<B>(w); break;
 
+#ifndef TP_UNIFORM_FASTPATH
+#define TP_UNIFORM_FASTPATH 1
+#endif
 __device__ __forceinline__ uint64_t sum_mb(const uint32_t* __restrict__ w, uint32_t b) {
   uint64_t r = 0;
+#if TP_UNIFORM_FASTPATH
+  const uint32_t bmin = __reduce_min_sync(FULL, b), bmax = __reduce_max_sync(FULL, b);
+  if (bmin == bmax) {
+    switch (bmin) {
+      TP_SCASE(0) TP_SCASE(1) TP_SCASE(2) TP_SCASE(3) TP_SCASE(4) TP_SCASE(5) TP_SCASE(6) TP_SCASE(7)
+      TP_SCASE(8) TP_SCASE(9) TP_SCASE(10) TP_SCASE(11) TP_SCASE(12) TP_SCASE(13) TP_SCASE(14) TP_SCASE(15)
+      TP_SCASE(16) TP_SCASE(17) TP_SCASE(18) TP_SCASE(19) TP_SCASE(20) TP_SCASE(21) TP_SCASE(22) TP_SCASE(23)
+      TP_SCASE(24) TP_SCASE(25) TP_SCASE(26) TP_SCASE(27) TP_SCASE(28) TP_SCASE(29) TP_SCASE(30) TP_SCASE(31)
+      default: r = sum_fixed<32>(w); break;
+    }
+    return r;
+  }
+#endif
   uint32_t todo = FULL;
   do {
     const uint32_t bl = __shfl_sync(FULL, b, __ffs(todo) - 1);

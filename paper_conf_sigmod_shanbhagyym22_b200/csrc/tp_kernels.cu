@@ -20,13 +20,11 @@ namespace tp {
 std::atomic<uint64_t> g_launches{0};
 
 // ------------------------------------------------------------------ stage context
-// A stage holds TPR * rounds consecutive tiles; consumers walk it in rounds of
-// TPR tiles (each consumer warp: 2 tiles = 32 miniblocks per round).
-constexpr uint32_t VIEW_WORDS = 4 * MAX_STREAMS;  // per-warp table: {lo, dshift, sshift, -} per stream
-
+// The ring holds "items": one column's words for a range of TPR * rounds consecutive
+// tiles.  Consumers walk a range in rounds of TPR tiles (each consumer warp: 2 tiles =
+// 32 miniblocks per round) and, within a round, the columns in evaluation order.
 struct StageCtx {
-  const uint32_t* stage;  // this stage's shared words
-  const uint32_t* views;  // the warp's per-stage stream table (see stage_views)
+  const uint32_t* stage;  // the current column item's shared words
   uint32_t t0s;           // first tile of the stage (global index)
   uint32_t round_base;    // stage-local index of the round's first tile
   uint32_t tile_end;      // one past the last tile of the CTA range
@@ -39,29 +37,17 @@ struct StreamView {
   uint32_t dshift, sshift;
 };
 
-// Computed once per stage by lane q for stream q (the stage's first copied word and
-// the 16-byte alignment shifts of the two bulk copies), read back by every decode.
-__device__ __forceinline__ void stage_views(const Params& P, uint32_t* views, const uint32_t* stage, uint32_t t0s,
-                                            uint32_t lane) {
-  if (lane < P.nstreams) {
-    const Stream& st = P.st[lane];
-    const uint32_t sidx = st.kind == K_RFOR ? t0s : 4u * t0s;
-    const uint32_t sshift = align_shift(st.starts, sidx);
-    const uint32_t lo = stage[st.starts_off + sshift] - (st.kind == K_DFOR ? 1u : 0u);
-    *reinterpret_cast<uint4*>(views + 4 * lane) = make_uint4(lo, align_shift(st.data, lo), sshift, 0u);
-  }
-  __syncwarp();
-}
-
+// Every lane derives the view itself (two smem loads + address arithmetic): cheaper on
+// the per-round critical path than sharing it through shared memory and a warp sync.
 __device__ __forceinline__ StreamView stream_view(const Params& P, uint32_t s, const StageCtx& C) {
   const Stream& st = P.st[s];
-  const uint4 t = *reinterpret_cast<const uint4*>(C.views + 4 * s);
   StreamView v;
+  const uint32_t sidx = st.kind == K_RFOR ? C.t0s : 4u * C.t0s;
   v.ss = C.stage + st.starts_off;
   v.sd = C.stage + st.data_off;
-  v.lo = t.x;
-  v.dshift = t.y;
-  v.sshift = t.z;
+  v.sshift = align_shift(st.starts, sidx);
+  v.lo = v.ss[v.sshift] - (st.kind == K_DFOR ? 1u : 0u);
+  v.dshift = align_shift(st.data, v.lo);
   return v;
 }
 
@@ -232,12 +218,17 @@ __device__ __forceinline__ void decode_col(const Params& P, uint32_t ci, const S
 }
 
 // ------------------------------------------------------------------ the pipeline
-// warp 0: TMA producer; warps 1..CONSUMER_WARPS: consumers (Op::stage per round).
+// warp 0: TMA producer; warps 1..CONSUMER_WARPS: consumers.  The item sequence is
+// (tile range g, column c) for g = 0.. and c = 0..ncols-1 in evaluation order, so a
+// query streams its columns one item at a time through a ring of small stages (a
+// multi-column tile does not have to fit shared memory at once).
+// Op interface: cta_init (all threads, before the first barrier), begin / col / end
+// per round of TPR tiles, finish (consumer warps, after their last round).
 template <class Op>
 __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
   extern __shared__ __align__(1024) uint32_t smem[];
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
-  const uint32_t TPS = TPR * P.rounds;  // tiles per stage
+  const uint32_t TPS = TPR * P.rounds;  // tiles per item
   // CTA tile range, in pairs of tiles so that a consumer warp's 1024 rows
   // never straddle two CTAs (decode->global stores whole warp boxes)
   const uint32_t npairs = (P.ntiles + 1u) >> 1;
@@ -245,9 +236,10 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
   const uint32_t p1 = (uint32_t)((uint64_t)(blockIdx.x + 1) * npairs / gridDim.x);
   const uint32_t t0 = 2u * p0, t1 = min(2u * p1, P.ntiles);
   if (t0 >= t1) return;
-  const uint32_t nst = (t1 - t0 + TPS - 1) / TPS;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + P.scratch_off + CONSUMER_WARPS * P.scratch_words_per_warp);
+  const uint32_t ngr = (t1 - t0 + TPS - 1) / TPS;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + P.bar_off);
   uint64_t* empty = full + P.nstages;
+  op.cta_init(P, smem);
   if (threadIdx.x == 0) {
     for (uint32_t s = 0; s < P.nstages; ++s) {
       mbar_init(&full[s], 1);
@@ -260,9 +252,10 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
   if (warp == 0) {
     // ---------------- producer
     const uint64_t pol = policy_evict_first();
-    for (uint32_t sb = 0; sb < nst; sb += 31) {
-      // lane i prefetches every stream's block_starts entry at the start of stage sb+i
-      const uint32_t tb = min(t0 + (sb + lane) * TPS, t1);
+    uint32_t slot = 0, phase = 0, item = 0;  // ring position of the next item (no runtime division)
+    for (uint32_t gb = 0; gb < ngr; gb += 31) {
+      // lane i prefetches every stream's block_starts entry at the start of range gb+i
+      const uint32_t tb = min(t0 + (gb + lane) * TPS, t1);
       uint32_t bnd[MAX_STREAMS];
 #pragma unroll
       for (int s = 0; s < MAX_STREAMS; ++s) {
@@ -273,77 +266,103 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
           bnd[s] = __ldg(st.starts + bi);
         }
       }
-      const uint32_t se = min(sb + 31, nst);
-      for (uint32_t s = sb; s < se; ++s) {
-        const uint32_t slot = s % P.nstages;
-        if (s >= P.nstages) mbar_wait_sleep(&empty[slot], ((s / P.nstages) + 1u) & 1u);
-        const uint32_t tile_base = t0 + s * TPS, tile_end = min(tile_base + TPS, t1);
-        uint32_t mylo = 0u, myhi = 0u;
+      const uint32_t ge = min(gb + 31, ngr);
+      for (uint32_t g = gb; g < ge; ++g) {
+        const uint32_t tile_base = t0 + g * TPS, tile_end = min(tile_base + TPS, t1);
+        for (uint32_t c = 0; c < P.ncols; ++c, ++item) {
+          if (item >= P.nstages) mbar_wait(&empty[slot], phase ^ 1u);
+          const Col& cc = P.col[c];
+          const uint32_t my_s = lane == 0 ? cc.s0 : (lane == 1 && cc.scheme == S_RFOR ? cc.s1 : 0xffu);
+          uint32_t mylo = 0u, myhi = 0u;
 #pragma unroll
-        for (int q = 0; q < MAX_STREAMS; ++q) {
-          if ((uint32_t)q < P.nstreams) {
-            const uint32_t a = __shfl_sync(FULL, bnd[q], s - sb);
-            const uint32_t b = __shfl_sync(FULL, bnd[q], s - sb + 1);
-            if (lane == (uint32_t)q) { mylo = a; myhi = b; }
+          for (int q = 0; q < MAX_STREAMS; ++q) {
+            if ((uint32_t)q < P.nstreams) {
+              const uint32_t a = __shfl_sync(FULL, bnd[q], g - gb);
+              const uint32_t b = __shfl_sync(FULL, bnd[q], g - gb + 1);
+              if (my_s == (uint32_t)q) { mylo = a; myhi = b; }
+            }
           }
-        }
-        uint32_t bytes = 0u;
-        const char *dsrc = nullptr, *ssrc = nullptr;
-        uint32_t dbytes = 0u, sbytes = 0u;
-        uint32_t* dst_d = nullptr;
-        uint32_t* dst_s = nullptr;
-        if (lane < P.nstreams) {
-          const Stream& st = P.st[lane];
-          const uint32_t lo = mylo - (st.kind == K_DFOR ? 1u : 0u);
-          const uintptr_t a0 = reinterpret_cast<uintptr_t>(st.data + lo) & ~uintptr_t(15);
-          const uintptr_t a1 = (reinterpret_cast<uintptr_t>(st.data + myhi) + 15) & ~uintptr_t(15);
-          dsrc = reinterpret_cast<const char*>(a0);
-          dbytes = (uint32_t)(a1 - a0);
-          const uint32_t s0 = st.kind == K_RFOR ? tile_base : 4u * tile_base;
-          const uint32_t s1 = min(st.kind == K_RFOR ? tile_end : 4u * tile_end, st.nblocks) + 1u;
-          const uintptr_t b0 = reinterpret_cast<uintptr_t>(st.starts + s0) & ~uintptr_t(15);
-          const uintptr_t b1 = (reinterpret_cast<uintptr_t>(st.starts + s1) + 15) & ~uintptr_t(15);
-          ssrc = reinterpret_cast<const char*>(b0);
-          sbytes = (uint32_t)(b1 - b0);
-          uint32_t* sbase = smem + slot * P.stage_words;
-          dst_d = sbase + st.data_off;
-          dst_s = sbase + st.starts_off;
-          bytes = dbytes + sbytes;
-        }
-        const uint32_t total = __reduce_add_sync(FULL, bytes);
-        if (lane == 0) mbar_arrive_expect_tx(&full[slot], total);
-        __syncwarp();
-        if (lane < P.nstreams) {
-          bulk_g2s(dst_d, dsrc, dbytes, &full[slot], pol);
-          bulk_g2s(dst_s, ssrc, sbytes, &full[slot], pol);
+          uint32_t bytes = 0u, dbytes = 0u, sbytes = 0u;
+          const char *dsrc = nullptr, *ssrc = nullptr;
+          uint32_t *dst_d = nullptr, *dst_s = nullptr;
+          if (my_s != 0xffu) {
+            const Stream& st = P.st[my_s];
+            const uint32_t lo = mylo - (st.kind == K_DFOR ? 1u : 0u);
+            const uintptr_t a0 = reinterpret_cast<uintptr_t>(st.data + lo) & ~uintptr_t(15);
+            const uintptr_t a1 = (reinterpret_cast<uintptr_t>(st.data + myhi) + 15) & ~uintptr_t(15);
+            dsrc = reinterpret_cast<const char*>(a0);
+            dbytes = (uint32_t)(a1 - a0);
+            const uint32_t s0 = st.kind == K_RFOR ? tile_base : 4u * tile_base;
+            const uint32_t s1 = min(st.kind == K_RFOR ? tile_end : 4u * tile_end, st.nblocks) + 1u;
+            const uintptr_t b0 = reinterpret_cast<uintptr_t>(st.starts + s0) & ~uintptr_t(15);
+            const uintptr_t b1 = (reinterpret_cast<uintptr_t>(st.starts + s1) + 15) & ~uintptr_t(15);
+            ssrc = reinterpret_cast<const char*>(b0);
+            sbytes = (uint32_t)(b1 - b0);
+            uint32_t* ibase = smem + slot * P.stage_words;
+            dst_d = ibase + st.data_off;
+            dst_s = ibase + st.starts_off;
+            bytes = dbytes + sbytes;
+          }
+          const uint32_t total = __reduce_add_sync(FULL, bytes);
+          if (lane == 0) mbar_arrive_expect_tx(&full[slot], total);
+          __syncwarp();
+          if (my_s != 0xffu) {
+            bulk_g2s(dst_d, dsrc, dbytes, &full[slot], pol);
+            bulk_g2s(dst_s, ssrc, sbytes, &full[slot], pol);
+          }
+          if (++slot == P.nstages) { slot = 0; phase ^= 1u; }
         }
       }
     }
   } else {
     // ---------------- consumers
     const Lane g = lane_geom();
-    uint32_t* views = smem + P.scratch_off + g.cw * P.scratch_words_per_warp;
-    uint32_t* scratch = views + VIEW_WORDS;
+    uint32_t* scratch = smem + P.scratch_off + g.cw * P.scratch_words_per_warp;
     uint32_t rc = 0;  // round counter (decode->global buffer parity)
-    for (uint32_t s = 0; s < nst; ++s) {
-      const uint32_t slot = s % P.nstages;
-      mbar_wait(&full[slot], (s / P.nstages) & 1u);
-      StageCtx C;
-      C.stage = smem + slot * P.stage_words;
-      C.views = views;
-      C.t0s = t0 + s * TPS;
-      stage_views(P, views, C.stage, C.t0s, g.lane);
-      C.tile_end = t1;
-      const uint32_t nr = min(P.rounds, (t1 - C.t0s + TPR - 1) / TPR);
-      for (uint32_t r = 0; r < nr; ++r, ++rc) {
-        C.round_base = r * TPR;
-        op.stage(P, C, g, scratch, rc);
+    uint32_t slot = 0, phase = 0;
+    StageCtx C;
+    C.tile_end = t1;
+    if (P.ncols == 1) {
+      // single column: one item per tile range, walked in P.rounds rounds
+      for (uint32_t gi = 0; gi < ngr; ++gi) {
+        C.t0s = t0 + gi * TPS;
+        C.stage = smem + slot * P.stage_words;
+        const uint32_t nr = min(P.rounds, (t1 - C.t0s + TPR - 1) / TPR);
+        mbar_wait(&full[slot], phase);
+        for (uint32_t r = 0; r < nr; ++r, ++rc) {
+          C.round_base = r * TPR;
+          op.begin(P, C, g);
+          op.col(P, C, g, scratch, 0, rc);
+          op.end(P, C, g);
+        }
+        __syncwarp();
+        if (g.lane == 0) mbar_arrive(&empty[slot]);
+        if (++slot == P.nstages) { slot = 0; phase ^= 1u; }
       }
-      __syncwarp();
-      if (g.lane == 0) mbar_arrive(&empty[slot]);
+    } else {
+      // queries: one round per tile range; the columns' items arrive in evaluation order
+      C.round_base = 0;
+      for (uint32_t gi = 0; gi < ngr; ++gi, ++rc) {
+        C.t0s = t0 + gi * TPS;
+        op.begin(P, C, g);
+        for (uint32_t c = 0; c < P.ncols; ++c) {
+          C.stage = smem + slot * P.stage_words;
+          mbar_wait(&full[slot], phase);
+          op.col(P, C, g, scratch, c, rc);
+          __syncwarp();
+          if (g.lane == 0) mbar_arrive(&empty[slot]);
+          if (++slot == P.nstages) { slot = 0; phase ^= 1u; }
+        }
+        op.end(P, C, g);
+      }
     }
-    op.finish(P, g);
+    op.finish(P, g, smem);
   }
+}
+
+// named barrier over the consumer warps only
+__device__ __forceinline__ void consumers_sync() {
+  asm volatile("bar.sync 1, %0;" ::"n"(CONSUMER_WARPS * 32) : "memory");
 }
 
 // ------------------------------------------------------------------ consumers
@@ -353,22 +372,35 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t x) {
   return x;
 }
 
+__device__ __forceinline__ uint32_t valid_rows(const Params& P, const StageCtx& C, const Lane& g) {
+  const uint32_t tile = C.t0s + C.round_base + g.tile_local;
+  const uint32_t row0 = tile * TILE_ROWS + g.mb * MB_ROWS;
+  if (tile >= C.tile_end || row0 >= P.n) return 0u;
+  const uint32_t nrows = P.n - row0;
+  return nrows >= 32u ? 0xffffffffu : ((1u << nrows) - 1u);
+}
+
+struct OpBase {
+  __device__ void cta_init(const Params&, uint32_t*) {}
+  __device__ void begin(const Params&, const StageCtx&, const Lane&) {}
+  __device__ void end(const Params&, const StageCtx&, const Lane&) {}
+};
+
 // decode -> sum (decode-only microbenchmark)
 template <uint32_t MASK>
-struct SumOp {
+struct SumOp : OpBase {
   unsigned long long* out;
   uint64_t acc;
-  __device__ void stage(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t) {
+  __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t, uint32_t) {
     const Col& c = P.col[0];
-    const uint32_t tile = C.t0s + C.round_base + g.tile_local;
-    const uint32_t row0 = tile * TILE_ROWS + g.mb * MB_ROWS;
-    const bool tv = tile < C.tile_end;
+    const uint32_t alive = valid_rows(P, C, g);
     if (MASK == M_FOR) {
       const StreamView v = stream_view(P, c.s0, C);
       uint32_t tl;
-      bool tv2;
-      const MbView m = for_mb(P, c, C, g, v, tl, tv2);
-      if (tv && row0 + MB_ROWS <= P.n) {
+      bool tv;
+      const MbView m = for_mb(P, c, C, g, v, tl, tv);
+      // the branch must be warp-uniform: both sides run warp-collective dispatch code
+      if (__all_sync(FULL, alive == 0xffffffffu)) {
         const uint64_t se = sum_mb(m.w, m.b);
         acc += se + (uint64_t)((int64_t)(int32_t)m.ref * 32);
       } else {
@@ -376,22 +408,17 @@ struct SumOp {
         unpack_mb(m.w, m.b, e);
 #pragma unroll
         for (int i = 0; i < 32; ++i)
-          if (tv && row0 + i < P.n) acc += (uint64_t)(int64_t)(int32_t)(m.ref + e[i]);
+          if (alive & (1u << i)) acc += (uint64_t)(int64_t)(int32_t)(m.ref + e[i]);
       }
     } else {
       uint32_t val[32];
       decode_col<MASK>(P, 0, C, g, scratch, val);
-      if (tv && row0 + MB_ROWS <= P.n) {
 #pragma unroll
-        for (int i = 0; i < 32; ++i) acc += (uint64_t)(int64_t)(int32_t)val[i];
-      } else {
-#pragma unroll
-        for (int i = 0; i < 32; ++i)
-          if (tv && row0 + i < P.n) acc += (uint64_t)(int64_t)(int32_t)val[i];
-      }
+      for (int i = 0; i < 32; ++i)
+        if (alive & (1u << i)) acc += (uint64_t)(int64_t)(int32_t)val[i];
     }
   }
-  __device__ void finish(const Params&, const Lane& g) {
+  __device__ void finish(const Params&, const Lane& g, uint32_t*) {
     const uint64_t s = warp_sum_u64(acc);
     if (g.lane == 0) atomicAdd(out, (unsigned long long)s);
   }
@@ -401,27 +428,26 @@ struct SumOp {
 // 128B-swizzled 4 KB shared buffer (conflict-free 16-byte stores) and leave by
 // one TMA tensor store; the partial last miniblock (n % 32 rows) is stored directly.
 template <uint32_t MASK>
-struct GlobalOp {
+struct GlobalOp : OpBase {
   const CUtensorMap* tmap;
   int32_t* out;
   uint32_t full_rows32;  // n / 32: rows of the [n/32][32] tensor
-  __device__ void stage(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t s) {
+  __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t,
+                      uint32_t rc) {
     uint32_t val[32];
     decode_col<MASK>(P, 0, C, g, scratch, val);
     const uint32_t pair_tile = C.t0s + C.round_base + 2u * g.cw;
     if (pair_tile >= C.tile_end) return;  // warp-uniform
-    // staging buffers: 2 x 4 KB per warp, 1024-aligned, after the RFOR scratch
     uint32_t* buf = scratch + P.staging_off;
     buf = reinterpret_cast<uint32_t*>((reinterpret_cast<uintptr_t>(buf) + 1023) & ~uintptr_t(1023));
-    buf += (s & 1u) * 1024u;
-    if (g.lane == 0) bulk_wait_read<1>();  // the store issued from this buffer two stages ago is done reading
+    buf += (rc & 1u) * 1024u;
+    if (g.lane == 0) bulk_wait_read<1>();  // the store issued from this buffer two rounds ago is done reading
     __syncwarp();
     const uint32_t l = g.lane;
 #pragma unroll
-    for (uint32_t q = 0; q < 8; ++q) {
+    for (uint32_t q = 0; q < 8; ++q)
       st_shared_v4(buf + l * 32u + ((q ^ (l & 7u)) << 2), val[4 * q], val[4 * q + 1], val[4 * q + 2],
                    val[4 * q + 3]);
-    }
     fence_proxy_async_smem();
     __syncwarp();
     const uint32_t mb0 = pair_tile * 16u;
@@ -436,82 +462,231 @@ struct GlobalOp {
         if (mym * 32u + i < P.n) out[mym * 32u + i] = (int32_t)val[i];
     }
   }
-  __device__ void finish(const Params&, const Lane& g) {
+  __device__ void finish(const Params&, const Lane& g, uint32_t*) {
     if (g.lane == 0) bulk_wait_all();
     __syncwarp();
   }
 };
 
-// select / project / aggregate over up to 6 columns.  The host orders
-// the columns predicate-only first, then the projection operands a and b, so that
-// at most two decoded miniblocks are live at a time.
+// select / project / aggregate over up to 6 columns.  The host hands
+// the columns over in evaluation order: predicate-only columns, then the projection
+// operands a and b, so that at most two decoded miniblocks are live at a time.
 struct SelectArgs {
-  int32_t lo[TP_MAX_COLS], hi[TP_MAX_COLS];  // per position in `order`
-  uint32_t order[TP_MAX_COLS];               // column index per position
-  uint32_t npred;                            // positions [0, npred) are predicate-only
+  int32_t lo[TP_MAX_COLS], hi[TP_MAX_COLS];  // per column (evaluation order)
+  uint32_t npred;                            // columns [0, npred) are predicate-only
   int proj;                                  // TP_PROJ_*
-  uint32_t has_a, has_b;                     // positions npred (a) and npred+1 (b) present
+  uint32_t has_a, has_b;                     // column npred is a, npred+1 is b
 };
 
 template <uint32_t MASK>
-struct SelectOp {
+struct SelectOp : OpBase {
   const SelectArgs* A;
   unsigned long long* out;
   uint64_t acc;
-  __device__ __forceinline__ void pred(uint32_t k, const uint32_t (&v)[32], uint32_t& alive) const {
-    const int32_t l = A->lo[k], h = A->hi[k];
+  uint32_t alive;
+  uint32_t va[32];
+  __device__ void begin(const Params& P, const StageCtx& C, const Lane& g) { alive = valid_rows(P, C, g); }
+  __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c, uint32_t) {
+    if (!__any_sync(FULL, alive != 0u)) return;  // nothing survives in this warp's rows
+    uint32_t v[32];
+    decode_col<MASK>(P, c, C, g, scratch, v);
+    const int32_t l = A->lo[c], h = A->hi[c];
 #pragma unroll
-    for (int i = 0; i < 32; ++i) {
-      const int32_t x = (int32_t)v[i];
-      if (x < l || x > h) alive &= ~(1u << i);
-    }
-  }
-  __device__ void stage(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t) {
-    const uint32_t tile = C.t0s + C.round_base + g.tile_local;
-    const uint32_t row0 = tile * TILE_ROWS + g.mb * MB_ROWS;
-    uint32_t alive = 0u;
-    if (tile < C.tile_end && row0 < P.n) {
-      const uint32_t nrows = P.n - row0;
-      alive = nrows >= 32u ? 0xffffffffu : ((1u << nrows) - 1u);
-    }
-    const uint32_t nk = A->npred + A->has_a + A->has_b;
-    const uint32_t ka = A->has_a ? A->npred : 0xffffffffu;
-    const uint32_t kb = A->has_b ? A->npred + 1u : 0xffffffffu;
-    const bool mul = A->proj == TP_PROJ_MUL;
-    uint32_t va[32];
-    for (uint32_t k = 0; k < nk; ++k) {  // one decode call site: keeps the kernel small
-      uint32_t v[32];
-      decode_col<MASK>(P, A->order[k], C, g, scratch, v);
-      pred(k, v, alive);
-      if (k == ka) {
-        if (A->has_b) {
+    for (int i = 0; i < 32; ++i)
+      if ((int32_t)v[i] < l || (int32_t)v[i] > h) alive &= ~(1u << i);
+    if (A->has_a && c == A->npred) {
+      if (A->has_b) {
 #pragma unroll
-          for (int i = 0; i < 32; ++i) va[i] = v[i];
-        } else {
+        for (int i = 0; i < 32; ++i) va[i] = v[i];
+      } else {
 #pragma unroll
-          for (int i = 0; i < 32; ++i)
-            if (alive & (1u << i)) acc += (uint64_t)(int64_t)(int32_t)v[i];
-        }
-      } else if (k == kb) {
+        for (int i = 0; i < 32; ++i)
+          if (alive & (1u << i)) acc += (uint64_t)(int64_t)(int32_t)v[i];
+      }
+    } else if (A->has_b && c == A->npred + 1) {
+      const bool mul = A->proj == TP_PROJ_MUL;
 #pragma unroll
-        for (int i = 0; i < 32; ++i) {
-          if (alive & (1u << i)) {
-            const int64_t xa = (int32_t)va[i], xb = (int32_t)v[i];
-            acc += (uint64_t)(mul ? xa * xb : xa - xb);
-          }
+      for (int i = 0; i < 32; ++i) {
+        if (alive & (1u << i)) {
+          const int64_t xa = (int32_t)va[i], xb = (int32_t)v[i];
+          acc += (uint64_t)(mul ? xa * xb : xa - xb);
         }
       }
     }
+  }
+  __device__ void end(const Params&, const StageCtx&, const Lane&) {
     if (A->proj == TP_PROJ_COUNT) acc += __popc(alive);
   }
-  __device__ void finish(const Params&, const Lane& g) {
+  __device__ void finish(const Params&, const Lane& g, uint32_t*) {
     const uint64_t s = warp_sum_u64(acc);
     if (g.lane == 0) atomicAdd(out, (unsigned long long)s);
   }
 };
 
+// ------------------------------------------------------------------ star-join queries
+// SSB as one tile kernel: FK columns probe dimension lookup tables
+// (Crystal's perfect hash, key - key_min), payloads build a dense group index,
+// measures are aggregated per group.  Columns come in the host's order: filters and
+// probes first (most selective first), measures last.  Grouped queries pre-aggregate
+// in a per-CTA shared-memory hash table (open addressing) and flush it once, so hot
+// groups (q4.1 has 35) do not serialise on global atomics.
+struct StarArgs {
+  int32_t role[TP_MAX_COLS], lo[TP_MAX_COLS], hi[TP_MAX_COLS];
+  const int32_t* table[TP_MAX_COLS];
+  int32_t key_min[TP_MAX_COLS];
+  uint32_t table_len[TP_MAX_COLS], stride[TP_MAX_COLS];
+  int agg;
+  uint32_t ngroups;
+  long long* sums;
+  unsigned long long* counts;
+};
+
+constexpr uint32_t HT_SLOTS = 2048, HT_EMPTY = 0xffffffffu, HT_PROBES = 64;
+constexpr uint32_t HT_WORDS = HT_SLOTS * 4;  // keys + sum lo + sum hi + counts, one word each per slot
+
+template <uint32_t MASK, bool GROUPED>
+struct StarOp : OpBase {
+  const StarArgs* A;
+  uint64_t acc, cnt;  // ungrouped (q1.x): reduce in registers
+  uint32_t alive, nmeas;
+  uint32_t gv[32];    // grouped: group index per row; ungrouped: first measure (MUL)
+  uint32_t* keys;
+  uint32_t* hlo;   // 64-bit sums as lo/hi words: native 32-bit shared atomics with a carry
+  uint32_t* hhi;   // (a 64-bit shared atomicAdd is a CAS loop on sm_100)
+  uint32_t* hcnt;
+
+  __device__ void cta_init(const Params& P, uint32_t* smem) {
+    if (GROUPED) {
+      keys = smem + P.agg_off;
+      hlo = keys + HT_SLOTS;
+      hhi = keys + 2 * HT_SLOTS;
+      hcnt = keys + 3 * HT_SLOTS;
+      for (uint32_t i = threadIdx.x; i < HT_SLOTS; i += blockDim.x) {
+        keys[i] = HT_EMPTY;
+        hlo[i] = 0u;
+        hhi[i] = 0u;
+        hcnt[i] = 0u;
+      }
+    }
+  }
+  __device__ __forceinline__ void add(uint32_t key, int64_t v, uint32_t k) {
+    uint32_t slot = (key * 0x9E3779B1u) >> 21;  // 11-bit multiplicative hash
+#pragma unroll 1
+    for (uint32_t p = 0; p < HT_PROBES; ++p) {
+      uint32_t cur = keys[slot];
+      if (cur == HT_EMPTY) {
+        cur = atomicCAS(&keys[slot], HT_EMPTY, key);
+        if (cur == HT_EMPTY) cur = key;
+      }
+      if (cur == key) {
+        const uint32_t lo = (uint32_t)(uint64_t)v, hi = (uint32_t)((uint64_t)v >> 32);
+        const uint32_t old = atomicAdd(&hlo[slot], lo);
+        const uint32_t carry = old + lo < old ? 1u : 0u;
+        if (hi + carry) atomicAdd(&hhi[slot], hi + carry);
+        if (k) atomicAdd(&hcnt[slot], k);
+        return;
+      }
+      slot = (slot + 1u) & (HT_SLOTS - 1u);
+    }
+    atomicAdd(reinterpret_cast<unsigned long long*>(A->sums) + key, (unsigned long long)v);  // table crowded
+    if (k) atomicAdd(A->counts + key, (unsigned long long)k);
+  }
+  __device__ void begin(const Params& P, const StageCtx& C, const Lane& g) {
+    alive = valid_rows(P, C, g);
+    nmeas = 0;
+    if (GROUPED) {
+#pragma unroll
+      for (int i = 0; i < 32; ++i) gv[i] = 0u;
+    }
+  }
+  __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c, uint32_t) {
+    const int role = A->role[c];
+    if (!__any_sync(FULL, alive != 0u)) {  // nothing survives in this warp's rows: skip the decode
+      if (role == TP_ROLE_MEASURE) ++nmeas;
+      return;
+    }
+    uint32_t v[32];
+    decode_col<MASK>(P, c, C, g, scratch, v);
+    if (role == TP_ROLE_PROBE) {
+      const int32_t* __restrict__ T = A->table[c];
+      const uint32_t kmin = (uint32_t)A->key_min[c], len = A->table_len[c], stride = A->stride[c];
+      // all 32 probes are issued before any result is used (the row mask is read from a
+      // snapshot, so no probe waits for the previous one: 32 L2 requests in flight)
+      const uint32_t m = alive;
+      int32_t pl[32];
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        const uint32_t k = v[i] - kmin;
+        pl[i] = ((m >> i) & 1u) && k < len ? __ldg(T + k) : -1;
+      }
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        if (pl[i] < 0) alive &= ~(1u << i);
+        else if (GROUPED) gv[i] += (uint32_t)pl[i] * stride;
+      }
+      return;
+    }
+    const int32_t l = A->lo[c], h = A->hi[c];  // RANGE, or the measure's own filter
+#pragma unroll
+    for (int i = 0; i < 32; ++i)
+      if ((int32_t)v[i] < l || (int32_t)v[i] > h) alive &= ~(1u << i);
+    if (role == TP_ROLE_RANGE) return;
+    // measure
+    if (GROUPED) {
+      const bool neg = nmeas == 1;  // TP_AGG_SUB's second measure (MUL is not grouped)
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        if (alive & (1u << i)) {
+          const int64_t x = (int32_t)v[i];
+          add(gv[i], neg ? -x : x, neg ? 0u : 1u);
+        }
+      }
+    } else if (nmeas == 0 && A->agg == TP_AGG_MUL) {
+#pragma unroll
+      for (int i = 0; i < 32; ++i) gv[i] = v[i];
+    } else {
+      const bool mul = A->agg == TP_AGG_MUL, neg = nmeas == 1 && A->agg == TP_AGG_SUB;
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        if (alive & (1u << i)) {
+          int64_t x = (int32_t)v[i];
+          if (mul) x *= (int64_t)(int32_t)gv[i];
+          acc += (uint64_t)(neg ? -x : x);
+        }
+      }
+    }
+    ++nmeas;
+  }
+  __device__ void end(const Params&, const StageCtx&, const Lane&) {
+    if (!GROUPED) cnt += __popc(alive);
+  }
+  __device__ void finish(const Params&, const Lane& g, uint32_t*) {
+    if (GROUPED) {
+      consumers_sync();
+      for (uint32_t i = threadIdx.x - 32u; i < HT_SLOTS; i += CONSUMER_WARPS * 32u) {
+        const uint32_t k = keys[i];
+        if (k != HT_EMPTY) {
+          atomicAdd(reinterpret_cast<unsigned long long*>(A->sums) + k,
+                    ((unsigned long long)hhi[i] << 32) | hlo[i]);
+          atomicAdd(A->counts + k, (unsigned long long)hcnt[i]);
+        }
+      }
+    } else {
+      const uint64_t s = warp_sum_u64(acc), k = warp_sum_u64(cnt);
+      if (g.lane == 0) {
+        atomicAdd(reinterpret_cast<unsigned long long*>(A->sums), (unsigned long long)s);
+        atomicAdd(A->counts, (unsigned long long)k);
+      }
+    }
+  }
+};
+
+// ------------------------------------------------------------------ kernels
+#ifndef TP_SUM_MINB
+#define TP_SUM_MINB 4
+#endif
 template <uint32_t MASK>
-__global__ void __launch_bounds__(THREADS, 4) k_decode_sum(const __grid_constant__ Params P, unsigned long long* out) {
+__global__ void __launch_bounds__(THREADS, TP_SUM_MINB) k_decode_sum(const __grid_constant__ Params P, unsigned long long* out) {
   SumOp<MASK> op;
   op.out = out;
   op.acc = 0;
@@ -529,13 +704,48 @@ __global__ void __launch_bounds__(THREADS, 4)
 }
 
 template <uint32_t MASK>
-__global__ void __launch_bounds__(THREADS, 2)
+__global__ void __launch_bounds__(THREADS, 3)
     k_select_sum(const __grid_constant__ Params P, const __grid_constant__ SelectArgs A, unsigned long long* out) {
   SelectOp<MASK> op;
   op.A = &A;
   op.out = out;
   op.acc = 0;
+  op.alive = 0;
   run_pipeline(P, op);
+}
+
+template <uint32_t MASK, bool GROUPED>
+__global__ void __launch_bounds__(THREADS, 3)
+    k_star_query(const __grid_constant__ Params P, const __grid_constant__ StarArgs A) {
+  StarOp<MASK, GROUPED> op;
+  op.A = &A;
+  op.acc = 0;
+  op.cnt = 0;
+  op.alive = 0;
+  op.nmeas = 0;
+  run_pipeline(P, op);
+}
+
+// dimension lookup tables (the hash-table build of Crystal's star joins)
+__global__ void k_fill(int32_t* __restrict__ t, uint32_t len, int32_t v) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < len; i += gridDim.x * blockDim.x) t[i] = v;
+}
+struct DimArgs {
+  tp_dim_pred pred[4];
+  int npreds;
+};
+__global__ void k_lookup_build(const int32_t* __restrict__ keys, uint32_t nrows, int32_t key_min, uint32_t len,
+                               const __grid_constant__ DimArgs D, const int32_t* __restrict__ payload,
+                               int32_t* __restrict__ table) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nrows; i += gridDim.x * blockDim.x) {
+    bool ok = true;
+    for (int p = 0; p < D.npreds; ++p) {
+      const int32_t a = D.pred[p].attr[i];
+      ok &= (a >= D.pred[p].lo1 && a <= D.pred[p].hi1) || (a >= D.pred[p].lo2 && a <= D.pred[p].hi2);
+    }
+    const uint32_t k = (uint32_t)(keys[i] - key_min);
+    if (ok && k < len) table[k] = payload ? payload[i] : 0;
+  }
 }
 
 // uncompressed int32 scan -> sum ("None"): the HBM read roof of the same consumer
@@ -568,14 +778,22 @@ static int sm_count() {
   return g_sms;
 }
 
+#ifndef TP_MAX_STAGES
+#define TP_MAX_STAGES 8
+#endif
+#ifndef TP_RING_KB
+#define TP_RING_KB 40
+#endif
 static uint32_t worst_tile_words(uint32_t scheme) {
   return scheme == TP_FOR ? 4u * (2u + 128u) : scheme == TP_DFOR ? 1u + 4u * (2u + 128u) : 6u + 512u;
 }
 static uint32_t align4(uint32_t w) { return (w + 3u) & ~3u; }
 
-// Validate columns and lay the stage out: per stream a data region
-// (TPS tiles of at most max_tile_words + alignment slop) and a block_starts region.
-static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_scratch,
+// Validate the columns and lay out one ring item: per stream of the item's column a
+// data region (TPR * rounds tiles of at most max_tile_words + alignment slop) and a
+// block_starts region; item size = the largest column's.  extra_scratch: words per
+// consumer warp (after the view table); agg_words: per-CTA aggregation table.
+static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_scratch, uint32_t agg_words,
                               Params& P, size_t& smem_bytes) {
   memset(&P, 0, sizeof(P));
   if (!cols || ncols < 1 || ncols > TP_MAX_COLS) return TP_EINVAL;
@@ -583,7 +801,7 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
   if (n >= (1ull << 32)) return TP_EUNSUPPORTED;
   bool any_rfor = false;
   uint32_t mtws[MAX_STREAMS];
-  uint32_t round_words = 0;  // data words of one round (TPR tiles) over all streams, upper bound
+  uint32_t max_round_words = 0;  // data words of one round (TPR tiles) of the widest column
   for (int c = 0; c < ncols; ++c) {
     const tp_column& k = cols[c];
     if (k.n != n) return TP_EINVAL;
@@ -602,6 +820,7 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
     Col& cc = P.col[c];
     cc.scheme = k.scheme == TP_FOR ? S_FOR : k.scheme == TP_DFOR ? S_DFOR : S_RFOR;
     cc.nblocks = (uint32_t)k.num_blocks;
+    uint32_t rw = 0;
     for (int s = 0; s < (rf ? 2 : 1); ++s) {
       Stream& st = P.st[P.nstreams];
       st.data = s == 0 ? k.data0 : k.data1;
@@ -611,38 +830,48 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
       uint32_t mtw = s == 0 ? k.max_tile_words0 : k.max_tile_words1;
       if (mtw == 0 || mtw > worst_tile_words(k.scheme)) mtw = worst_tile_words(k.scheme);
       mtws[P.nstreams] = mtw;
-      round_words += TPR * mtw;
+      rw += TPR * mtw;
       if (s == 0) cc.s0 = P.nstreams; else cc.s1 = P.nstreams;
       ++P.nstreams;
     }
+    max_round_words = std::max(max_round_words, rw);
   }
-  // rounds per stage: a stage carries ~16 KB of compressed words (bytes in flight for
-  // low bitwidths, where a round of 8 tiles is only a few hundred bytes), at most 8 rounds
+  // rounds per item: single-column kernels carry ~16 KB of compressed words per item
+  // (bytes in flight at low bitwidths, where one round is a few hundred bytes); queries
+  // keep per-round row state across columns, so they use one round per item
   const uint32_t target_words = 4096;
-  P.rounds = std::max<uint32_t>(1u, std::min<uint32_t>(8u, target_words / std::max<uint32_t>(round_words, 1u)));
+  P.rounds = ncols > 1 ? 1u
+                       : std::max<uint32_t>(1u, std::min<uint32_t>(8u, target_words / std::max(max_round_words, 1u)));
   const uint32_t TPS = TPR * P.rounds;
-  uint32_t off = 0;
-  for (uint32_t q = 0; q < P.nstreams; ++q) {
-    Stream& st = P.st[q];
-    st.data_off = off;
-    off += align4(std::max<uint32_t>(TPS * mtws[q] + 12u, 48u));  // + alignment slop + unpack over-read
-    st.starts_off = off;
-    off += align4((st.kind == K_RFOR ? TPS + 1u : 4u * TPS + 1u) + 8u);
+  uint32_t item = 0;
+  for (int c = 0; c < ncols; ++c) {
+    uint32_t off = 0;
+    const uint32_t q0 = P.col[c].s0, q1 = P.col[c].scheme == S_RFOR ? P.col[c].s1 : q0;
+    for (uint32_t q = q0; q <= q1; ++q) {
+      Stream& st = P.st[q];
+      st.data_off = off;
+      off += align4(std::max<uint32_t>(TPS * mtws[q] + 12u, 48u));  // + alignment slop + unpack over-read
+      st.starts_off = off;
+      off += align4((st.kind == K_RFOR ? TPS + 1u : 4u * TPS + 1u) + 8u);
+    }
+    item = std::max(item, off);
   }
   P.ncols = (uint32_t)ncols;
   P.n = (uint32_t)n;
   P.ntiles = (uint32_t)((n + TILE_ROWS - 1) / TILE_ROWS);
-  P.stage_words = align4(off);
-  P.staging_off = any_rfor ? RFOR_SCRATCH_WORDS : 0u;  // relative to the scratch after the view table
-  const uint32_t scratch = VIEW_WORDS + P.staging_off + extra_scratch;
-  P.scratch_words_per_warp = align4(scratch);
-  // ring depth: 2..6 stages within ~40 KB so that 4+ CTAs (16+ consumer warps) fit an SM;
-  // 4 CTAs x 40 KB keeps ~100+ KB of TMA traffic in flight per SM
-  uint32_t nstg = 6;
-  while (nstg > 2 && (size_t)nstg * P.stage_words * 4 > 40 * 1024) --nstg;
+  P.stage_words = align4(item);
+  P.staging_off = any_rfor ? RFOR_SCRATCH_WORDS : 0u;
+  P.scratch_words_per_warp = align4(P.staging_off + extra_scratch);
+  // ring depth: 2..8 items within ~40 KB, so that several CTAs (16+ consumer warps) share
+  // an SM while ~100+ KB of TMA traffic stays in flight per SM
+  uint32_t nstg = TP_MAX_STAGES;
+  while (nstg > 2 && (size_t)nstg * P.stage_words * 4 > TP_RING_KB * 1024) --nstg;
   P.nstages = nstg;
   P.scratch_off = nstg * P.stage_words;
-  smem_bytes = (size_t)(P.scratch_off + CONSUMER_WARPS * P.scratch_words_per_warp) * 4 + 2 * nstg * 8 + 16;
+  P.agg_off = P.scratch_off + CONSUMER_WARPS * P.scratch_words_per_warp;
+  P.bar_off = align4(P.agg_off + agg_words);
+  if (P.bar_off & 1u) ++P.bar_off;  // 8-byte aligned barriers
+  smem_bytes = (size_t)P.bar_off * 4 + 2 * nstg * 8 + 16;
   return TP_OK;
 }
 
@@ -685,6 +914,17 @@ static PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
   return fn;
 }
 
+#define TP_DISPATCH_MASK(MASKV, CALL)                               \
+  switch (MASKV) {                                                  \
+    case M_FOR: { constexpr uint32_t MK = M_FOR; CALL; } break;     \
+    case M_DFOR: { constexpr uint32_t MK = M_DFOR; CALL; } break;   \
+    case M_RFOR: { constexpr uint32_t MK = M_RFOR; CALL; } break;   \
+    case M_FOR | M_DFOR: { constexpr uint32_t MK = M_FOR | M_DFOR; CALL; } break; \
+    case M_FOR | M_RFOR: { constexpr uint32_t MK = M_FOR | M_RFOR; CALL; } break; \
+    case M_DFOR | M_RFOR: { constexpr uint32_t MK = M_DFOR | M_RFOR; CALL; } break; \
+    default: { constexpr uint32_t MK = M_FOR | M_DFOR | M_RFOR; CALL; } break; \
+  }
+
 }  // namespace tp
 
 using namespace tp;
@@ -696,7 +936,7 @@ tp_status tp_decode_sum(const tp_column* dcol, int64_t* d_sum, void* stream) {
   if (dcol->n == 0) return TP_OK;
   Params P;
   size_t smem = 0;
-  tp_status st = build_params(dcol, 1, 0, P, smem);
+  tp_status st = build_params(dcol, 1, 0, 0, P, smem);
   if (st != TP_OK) return st;
   auto out = reinterpret_cast<unsigned long long*>(d_sum);
   const int cap = (int)((P.ntiles + 1) / 2);
@@ -714,8 +954,8 @@ tp_status tp_decode(const tp_column* dcol, int32_t* d_out, void* stream) {
   if (reinterpret_cast<uintptr_t>(d_out) & 15u) return TP_EINVAL;
   Params P;
   size_t smem = 0;
-  // per warp: RFOR scratch + 2 x 4 KB swizzled staging + 1 KB alignment slop
-  tp_status st = build_params(dcol, 1, 2048u + 256u, P, smem);
+  // per warp: 2 x 4 KB swizzled staging + 1 KB alignment slop
+  tp_status st = build_params(dcol, 1, 2048u + 256u, 0, P, smem);
   if (st != TP_OK) return st;
   CUtensorMap tmap;
   memset(&tmap, 0, sizeof(tmap));
@@ -748,35 +988,96 @@ tp_status tp_select_project_sum(const tp_column* dcols, int ncols, const int32_t
   if (proj_op != TP_PROJ_COUNT && (a < 0 || a >= ncols)) return TP_EINVAL;
   if ((proj_op == TP_PROJ_MUL || proj_op == TP_PROJ_SUB) && (b < 0 || b >= ncols)) return TP_EINVAL;
   if (dcols[0].n == 0) return TP_OK;
-  Params P;
-  size_t smem = 0;
-  tp_status st = build_params(dcols, ncols, 0, P, smem);
-  if (st != TP_OK) return st;
+  // evaluation order: predicate-only columns first, then a, then b (a == b decodes twice;
+  // predicates are idempotent)
+  const bool use_a = proj_op != TP_PROJ_COUNT, use_b = proj_op == TP_PROJ_MUL || proj_op == TP_PROJ_SUB;
+  tp_column ord[TP_MAX_COLS + 1];
   SelectArgs A;
   memset(&A, 0, sizeof(A));
   A.proj = proj_op;
-  const bool use_a = proj_op != TP_PROJ_COUNT, use_b = proj_op == TP_PROJ_MUL || proj_op == TP_PROJ_SUB;
-  uint32_t k = 0;
-  for (int c = 0; c < ncols; ++c) {  // predicate-only columns first
+  int k = 0;
+  for (int c = 0; c < ncols; ++c) {
     if ((use_a && c == a) || (use_b && c == b)) continue;
-    A.order[k] = (uint32_t)c; A.lo[k] = lo[c]; A.hi[k] = hi[c]; ++k;
+    ord[k] = dcols[c]; A.lo[k] = lo[c]; A.hi[k] = hi[c]; ++k;
   }
-  A.npred = k;
-  if (use_a) { A.order[k] = (uint32_t)a; A.lo[k] = lo[a]; A.hi[k] = hi[a]; ++k; A.has_a = 1; }
+  A.npred = (uint32_t)k;
+  if (use_a) { ord[k] = dcols[a]; A.lo[k] = lo[a]; A.hi[k] = hi[a]; ++k; A.has_a = 1; }
   if (use_b) {
-    // a == b (e.g. sum of squares) decodes the column twice; predicates are idempotent
-    A.order[k] = (uint32_t)b; A.lo[k] = lo[b]; A.hi[k] = hi[b]; ++k; A.has_b = 1;
+    if (k >= TP_MAX_COLS) return TP_EINVAL;
+    ord[k] = dcols[b]; A.lo[k] = lo[b]; A.hi[k] = hi[b]; ++k; A.has_b = 1;
   }
+  Params P;
+  size_t smem = 0;
+  tp_status st = build_params(ord, k, 0, 0, P, smem);
+  if (st != TP_OK) return st;
   auto out = reinterpret_cast<unsigned long long*>(d_result);
   const int cap = (int)((P.ntiles + 1) / 2);
-  switch (scheme_mask(P)) {
-    case M_FOR: launch(k_select_sum<M_FOR>, smem, cap, stream, P, A, out); break;
-    case M_DFOR: launch(k_select_sum<M_DFOR>, smem, cap, stream, P, A, out); break;
-    case M_RFOR: launch(k_select_sum<M_RFOR>, smem, cap, stream, P, A, out); break;
-    case M_FOR | M_DFOR: launch(k_select_sum<M_FOR | M_DFOR>, smem, cap, stream, P, A, out); break;
-    case M_FOR | M_RFOR: launch(k_select_sum<M_FOR | M_RFOR>, smem, cap, stream, P, A, out); break;
-    case M_DFOR | M_RFOR: launch(k_select_sum<M_DFOR | M_RFOR>, smem, cap, stream, P, A, out); break;
-    default: launch(k_select_sum<M_FOR | M_DFOR | M_RFOR>, smem, cap, stream, P, A, out); break;
+  TP_DISPATCH_MASK(scheme_mask(P), launch(k_select_sum<MK>, smem, cap, stream, P, A, out));
+  return launched();
+}
+
+tp_status tp_lookup_build(const int32_t* d_keys, uint64_t nrows, int32_t key_min, uint32_t table_len,
+                          const tp_dim_pred* preds, int npreds, const int32_t* d_payload, int32_t* d_table,
+                          void* stream) {
+  if (!d_table || (nrows && !d_keys) || npreds < 0 || npreds > 4 || (npreds && !preds)) return TP_EINVAL;
+  if (nrows >= (1ull << 32)) return TP_EUNSUPPORTED;
+  DimArgs D;
+  memset(&D, 0, sizeof(D));
+  for (int p = 0; p < npreds; ++p) {
+    if (!preds[p].attr) return TP_EINVAL;
+    D.pred[p] = preds[p];
+  }
+  D.npreds = npreds;
+  const int grid = sm_count() * 4;
+  k_fill<<<grid, 256, 0, (cudaStream_t)stream>>>(d_table, table_len, -1);
+  tp_status st = launched();
+  if (st != TP_OK || nrows == 0) return st;
+  k_lookup_build<<<grid, 256, 0, (cudaStream_t)stream>>>(d_keys, (uint32_t)nrows, key_min, table_len, D, d_payload,
+                                                         d_table);
+  return launched();
+}
+
+tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int ncols, int agg, int64_t* d_sums,
+                        uint64_t* d_counts, uint32_t ngroups, void* stream) {
+  if (!dcols || !roles || !d_sums || !d_counts || ncols < 1 || ncols > TP_MAX_COLS || ngroups < 1) return TP_EINVAL;
+  if (agg < TP_AGG_SUM || agg > TP_AGG_SUB) return TP_EINVAL;
+  if (agg == TP_AGG_MUL && ngroups > 1) return TP_EUNSUPPORTED;  // products are aggregated ungrouped (q1.x)
+  int nmeas = 0;
+  for (int c = 0; c < ncols; ++c) {
+    const tp_star_col& r = roles[c];
+    if (r.role < TP_ROLE_RANGE || r.role > TP_ROLE_MEASURE) return TP_EINVAL;
+    if (r.role == TP_ROLE_PROBE && (!r.table || r.table_len == 0)) return TP_EINVAL;
+    if (r.role == TP_ROLE_MEASURE) {
+      // with SUB the first measure's contribution is added before the second is read
+      if (nmeas == 1 && agg == TP_AGG_SUB && (r.lo != INT_MIN || r.hi != INT_MAX)) return TP_EINVAL;
+      ++nmeas;
+    } else if (nmeas) {
+      return TP_EINVAL;  // measures come last
+    }
+  }
+  if (nmeas != (agg == TP_AGG_SUM ? 1 : 2)) return TP_EINVAL;
+  if (dcols[0].n == 0) return TP_OK;
+  const bool grouped = ngroups > 1;
+  Params P;
+  size_t smem = 0;
+  tp_status st = build_params(dcols, ncols, 0, grouped ? HT_WORDS : 0u, P, smem);
+  if (st != TP_OK) return st;
+  StarArgs A;
+  memset(&A, 0, sizeof(A));
+  for (int c = 0; c < ncols; ++c) {
+    A.role[c] = roles[c].role; A.lo[c] = roles[c].lo; A.hi[c] = roles[c].hi;
+    A.table[c] = roles[c].table; A.key_min[c] = roles[c].key_min;
+    A.table_len[c] = roles[c].table_len; A.stride[c] = roles[c].stride;
+  }
+  A.agg = agg;
+  A.ngroups = ngroups;
+  A.sums = reinterpret_cast<long long*>(d_sums);
+  A.counts = reinterpret_cast<unsigned long long*>(d_counts);
+  const int cap = (int)((P.ntiles + 1) / 2);
+  if (grouped) {
+    TP_DISPATCH_MASK(scheme_mask(P), (launch(k_star_query<MK, true>, smem, cap, stream, P, A)));
+  } else {
+    TP_DISPATCH_MASK(scheme_mask(P), (launch(k_star_query<MK, false>, smem, cap, stream, P, A)));
   }
   return launched();
 }
@@ -800,9 +1101,10 @@ tp_status tp_device_info(int* sms, int* ctas_per_sm) {
     memset(&c, 0, sizeof(c));
     c.scheme = TP_FOR; c.block_size = 128; c.miniblock_count = 4; c.n = 1 << 20; c.num_blocks = (1 << 20) / 128;
     c.starts0 = reinterpret_cast<const uint32_t*>(16); c.data0 = c.starts0;
+    c.max_tile_words0 = 4 * (2 + 4 * 16);  // the bench column (b = 16)
     Params P;
     size_t smem = 0;
-    build_params(&c, 1, 0, P, smem);
+    build_params(&c, 1, 0, 0, P, smem);
     *ctas_per_sm = grid_for(k_decode_sum<M_FOR>, smem) / sm_count();
   }
   return TP_OK;

@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libtilepack.so")
+LIB_PATH = os.environ.get("TILEPACK_LIB_OVERRIDE") or os.path.join(_HERE, "libtilepack.so")  # override: A/B builds
 GUARD_WORDS = 4
 
 TP_FOR, TP_DFOR, TP_RFOR = 1, 2, 3
@@ -46,6 +46,21 @@ class tp_column(ctypes.Structure):
     ]
 
 
+class tp_dim_pred(ctypes.Structure):
+    _fields_ = [("attr", ctypes.c_void_p), ("lo1", ctypes.c_int32), ("hi1", ctypes.c_int32),
+                ("lo2", ctypes.c_int32), ("hi2", ctypes.c_int32)]
+
+
+class tp_star_col(ctypes.Structure):
+    _fields_ = [("role", ctypes.c_int32), ("lo", ctypes.c_int32), ("hi", ctypes.c_int32),
+                ("table", ctypes.c_void_p), ("key_min", ctypes.c_int32), ("table_len", ctypes.c_uint32),
+                ("stride", ctypes.c_uint32)]
+
+
+TP_ROLE_RANGE, TP_ROLE_PROBE, TP_ROLE_MEASURE = 0, 1, 2
+TP_AGG = {"sum": 0, "mul": 1, "sub": 2}
+
+
 def _load():
     if not os.path.exists(LIB_PATH):
         raise ImportError(
@@ -64,11 +79,15 @@ def _load():
         "tp_decode_sum": (i32, [colp, vp, vp]),
         "tp_select_project_sum": (i32, [colp, i32, vp, vp, i32, i32, i32, vp, vp]),
         "tp_plain_sum": (i32, [vp, u64, vp, vp]),
+        "tp_lookup_build": (i32, [vp, u64, ctypes.c_int32, u32, ctypes.POINTER(tp_dim_pred), i32, vp, vp, vp]),
+        "tp_star_query": (i32, [colp, ctypes.POINTER(tp_star_col), i32, i32, vp, vp, u32, vp]),
         "tp_status_string": (ctypes.c_char_p, [i32]),
         "tp_launch_count": (u64, []),
         "tp_device_info": (i32, [vp, vp]),
     }
     for name, (res, args) in sig.items():
+        if os.environ.get("TILEPACK_LIB_OVERRIDE") and not hasattr(L, name):
+            continue  # A/B experiments with older builds
         f = getattr(L, name)
         f.restype = res
         f.argtypes = args
@@ -148,6 +167,24 @@ def tp_select_project_sum(dcols, lo, hi, proj_op: int, a: int, b: int, d_result,
     hi = np.ascontiguousarray(hi, np.int32)
     _check(_lib.tp_select_project_sum(arr, n, _ptr(lo), _ptr(hi), proj_op, a, b, _ptr(d_result), _stream(stream)),
            "tp_select_project_sum")
+
+
+def tp_lookup_build(d_keys, nrows: int, key_min: int, table_len: int, preds, d_payload, d_table, stream=None):
+    """preds: list of (attr_tensor, lo1, hi1[, lo2, hi2])"""
+    arr = (tp_dim_pred * max(1, len(preds)))()
+    for i, p in enumerate(preds):
+        lo2, hi2 = (p[3], p[4]) if len(p) > 3 else (1, 0)
+        arr[i] = tp_dim_pred(_ptr(p[0]), p[1], p[2], lo2, hi2)
+    _check(_lib.tp_lookup_build(_ptr(d_keys), nrows, key_min, table_len, arr, len(preds), _ptr(d_payload),
+                                _ptr(d_table), _stream(stream)), "tp_lookup_build")
+
+
+def tp_star_query(dcols, roles, agg: int, d_sums, d_counts, ngroups: int, stream=None):
+    n = len(dcols)
+    carr = (tp_column * n)(*dcols)
+    rarr = (tp_star_col * n)(*roles)
+    _check(_lib.tp_star_query(carr, rarr, n, agg, _ptr(d_sums), _ptr(d_counts), ngroups, _stream(stream)),
+           "tp_star_query")
 
 
 def tp_plain_sum(d_x, n: int, d_sum, stream=None):
