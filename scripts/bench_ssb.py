@@ -42,9 +42,8 @@ def main():
     t0 = time.time()
     db = gen.generate(args.sf, seed=5000)
     n = len(db["lineorder"]["lo_orderdate"])
-    ntiles = (n + 511) // 512
-    r0 = 512 * (ntiles * rank // world)
-    r1 = min(n, 512 * (ntiles * (rank + 1) // world))
+    from paper_conf_sigmod_shanbhagyym22_b200.dist import tile_range
+    r0, r1 = tile_range(n, rank, world)
     gen_s = time.time() - t0
     eng = SSBEngine(db, dev, rows=(r0, r1))
     setup_s = time.time() - t0

@@ -125,3 +125,23 @@ def test_bench_size_for_b16_sampled():
     assert np.array_equal(got, x[idx])
     tail = out[n - 1000:].cpu().numpy()
     assert np.array_equal(tail, oracle.for_decode_range(e, n - 1000, n, dg))
+
+
+@pytest.mark.parametrize("scheme", SCHEMES)
+def test_fake_multi_gpu_shards(scheme):
+    """shard into k tile ranges, decode each shard on GPU 0, the pieces
+    concatenate to the column and the shard sums add up to the whole-column sum."""
+    from paper_conf_sigmod_shanbhagyym22_b200 import dist as tpd
+    n = 512 * 301 + 77
+    x = {"for": datagen.uniform_bits(20, n, seed=1), "dfor": datagen.sorted_uniform(n, seed=2),
+         "rfor": datagen.runs(n, 5, seed=3)}[scheme]
+    h = tp.encode(x, scheme)
+    for world in (2, 3, 8):
+        acc = torch.zeros(1, dtype=torch.int64, device="cuda")
+        pieces = []
+        for r in range(world):
+            d = tpd.shard(h, r, world).to_device()
+            pieces.append(tp.decode(d).cpu().numpy())
+            tp.decode_sum(d, out=acc)
+        assert np.array_equal(np.concatenate(pieces), x)
+        assert int(acc.item()) == oracle.column_sum(x)
