@@ -145,6 +145,24 @@ __device__ __forceinline__ uint32_t extract_lane(const uint32_t* m, uint32_t lan
   return __funnelshift_r(w[0], w[1], p) & mask;  // the funnel shift uses p mod 32
 }
 
+__device__ __forceinline__ uint32_t byte_of(const uint4& w, uint32_t m) {  // byte m (0..15)
+  const uint32_t q = m >> 2;
+  const uint32_t x = q == 0 ? w.x : q == 1 ? w.y : q == 2 ? w.z : w.w;
+  return (x >> (8u * (m & 3u))) & 255u;
+}
+__device__ __forceinline__ uint32_t bytes_before(const uint4& w, uint32_t m) {  // sum of bytes [0, m)
+  const uint32_t q = m >> 2;
+  const uint32_t sx = (w.x * 0x01010101u) >> 24, sy = (w.y * 0x01010101u) >> 24, sz = (w.z * 0x01010101u) >> 24;
+  const uint32_t full = (q > 0 ? sx : 0u) + (q > 1 ? sy : 0u) + (q > 2 ? sz : 0u);
+  const uint32_t x = q == 0 ? w.x : q == 1 ? w.y : q == 2 ? w.z : w.w;
+  return full + bw_prefix(x, m & 3u);
+}
+// b-bit field at stream bit p of m (p's word and the next one; the funnel shift uses p mod 32)
+__device__ __forceinline__ uint32_t extract_at(const uint32_t* m, uint32_t p, uint32_t mask) {
+  const uint32_t* w = m + (p >> 5);
+  return __funnelshift_r(w[0], w[1], p) & mask;
+}
+
 __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                             uint32_t* scratch, uint32_t (&val)[32]) {
   const StreamView vv = stream_view(P, c.s0, C), vl = stream_view(P, c.s1, C);
@@ -161,32 +179,52 @@ __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const
     const uint32_t* bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
     const uint32_t* bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
     const uint32_t r = min(bV[0], 512u);  // run / value count
-    const uint32_t nq = (r + 31u) >> 5;
     const uint32_t refV = bV[1], refL = bL[1];  // references (FOR on both arrays)
-    const uint8_t* bwV = reinterpret_cast<const uint8_t*>(bV + 2);  // bitwidth byte q = miniblock q (R2, R17)
-    const uint8_t* bwL = reinterpret_cast<const uint8_t*>(bL + 2);
-    const uint32_t* mV = bV + 6;  // [r][ref][4 bitwidth words] then the tight miniblocks (R17)
-    const uint32_t* mL = bL + 6;
+    // 4 bitwidth words per stream: byte m = miniblock m (R2, R17)
+    const uint4 wv = make_uint4(bV[2], bV[3], bV[4], bV[5]);  // 4-byte aligned only: scalar loads
+    const uint4 wl = make_uint4(bL[2], bL[3], bL[4], bL[5]);
     uint32_t carry = 0u;
-    for (uint32_t q = 0; q < nq; ++q) {  // one miniblock (32 entries) of each stream per step
-      const uint32_t bv = min((uint32_t)bwV[q], 32u), bl = min((uint32_t)bwL[q], 32u);
+    // lane l takes entries 128q + 4l .. 128q + 4l + 3 of both streams: all four sit in
+    // miniblock 4q + l/8 (one bitwidth, and all earlier miniblocks are full, R17)
+    for (uint32_t q = 0; 128u * q < r; ++q) {
+      const uint32_t m = 4u * q + (lane >> 3);
+      const uint32_t e0 = 128u * q + 4u * lane;
+      const uint32_t bv = min(byte_of(wv, m), 32u), bl = min(byte_of(wl, m), 32u);
       const uint32_t mv = __funnelshift_lc(0xffffffffu, 0u, bv), ml = __funnelshift_lc(0xffffffffu, 0u, bl);
-      const uint32_t e = 32u * q + lane;
-      const bool in = e < r;
-      // 1. lane-per-entry unpack (warp-uniform bitwidth per miniblock)
-      const uint32_t xv = refV + extract_lane(mV, lane, bv, mv);
-      const uint32_t xl = in ? refL + extract_lane(mL, lane, bl, ml) : 0u;
-      // 2. scan of the run lengths -> run start rows
-      const uint32_t incl = warp_inclusive_scan(xl, lane);
-      const uint32_t S = carry + incl - xl;
-      // 3. scatter the value and the run-start bit
-      if (in) {
-        V[e] = xv;
-        atomicOr(&bitmap[(S >> 5) & 15u], 1u << (S & 31u));
+      const uint32_t* mV = bV + 6 + bytes_before(wv, m);  // miniblock m's first word
+      const uint32_t* mL = bL + 6 + bytes_before(wl, m);
+      const uint32_t pos = 4u * (lane & 7u);
+      uint32_t xv[4], len[4], incl[4];
+      uint32_t run = 0u;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {  // 1. unpack + local inclusive scan of the lengths
+        const bool in = e0 + k < r;
+        xv[k] = refV + extract_at(mV, (pos + k) * bv, mv);
+        len[k] = in ? refL + extract_at(mL, (pos + k) * bl, ml) : 0u;
+        run += len[k];
+        incl[k] = run;
       }
-      carry += __shfl_sync(FULL, incl, 31);
-      mV += bv;  // full miniblocks occupy b words; only the last one can be partial
-      mL += bl;
+      // 2. warp scan of the per-lane totals -> run start rows
+      const uint32_t wincl = warp_inclusive_scan(run, lane);
+      const uint32_t base = carry + wincl - run;
+      // 3. scatter values and run-start bits (the 4 starts of a lane share at most a few words)
+      uint32_t cw = 0xffffffffu, cb = 0u;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        if (e0 + k < r) {
+          const uint32_t S = base + incl[k] - len[k];
+          V[e0 + k] = xv[k];
+          const uint32_t w = (S >> 5) & 15u;
+          if (w != cw) {
+            if (cb) atomicOr(&bitmap[cw], cb);
+            cw = w;
+            cb = 0u;
+          }
+          cb |= 1u << (S & 31u);
+        }
+      }
+      if (cb) atomicOr(&bitmap[cw], cb);
+      carry += __shfl_sync(FULL, wincl, 31);
     }
   }
   __syncwarp();
@@ -199,8 +237,10 @@ __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const
   const int before = (int)(seg16_inclusive_scan(pc) - pc);  // run starts before row 32j
 #pragma unroll
   for (int i = 0; i < 32; ++i) {
+    // row 0 of a row block always starts a run, so cur >= 0 for real rows; rows of a missing
+    // row block (no runs) read V[-1] = bitmap[15] -- in bounds, and masked by the consumer
     const int cur = before - 1 + __popc(bm & (0xffffffffu >> (31 - i)));
-    val[i] = V[cur < 0 ? 0 : cur];
+    val[i] = V[cur];
   }
   __syncwarp();
 }
@@ -270,7 +310,7 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
       for (uint32_t g = gb; g < ge; ++g) {
         const uint32_t tile_base = t0 + g * TPS, tile_end = min(tile_base + TPS, t1);
         for (uint32_t c = 0; c < P.ncols; ++c, ++item) {
-          if (item >= P.nstages) mbar_wait(&empty[slot], phase ^ 1u);
+          if (item >= P.nstages) mbar_wait_backoff(&empty[slot], phase ^ 1u);
           const Col& cc = P.col[c];
           const uint32_t my_s = lane == 0 ? cc.s0 : (lane == 1 && cc.scheme == S_RFOR ? cc.s1 : 0xffu);
           uint32_t mylo = 0u, myhi = 0u;
@@ -413,9 +453,20 @@ struct SumOp : OpBase {
     } else {
       uint32_t val[32];
       decode_col<MASK>(P, 0, C, g, scratch, val);
+      if (alive == 0xffffffffu) {  // per-lane branch, no collectives inside
+        uint64_t lo = 0;
+        uint32_t neg = 0;
 #pragma unroll
-      for (int i = 0; i < 32; ++i)
-        if (alive & (1u << i)) acc += (uint64_t)(int64_t)(int32_t)val[i];
+        for (int i = 0; i < 32; ++i) {  // sum(sext v) = sum(zext v) - 2^32 * #negative
+          lo += val[i];
+          neg += val[i] >> 31;
+        }
+        acc += lo - ((uint64_t)neg << 32);
+      } else {
+#pragma unroll
+        for (int i = 0; i < 32; ++i)
+          if (alive & (1u << i)) acc += (uint64_t)(int64_t)(int32_t)val[i];
+      }
     }
   }
   __device__ void finish(const Params&, const Lane& g, uint32_t*) {
@@ -537,12 +588,19 @@ struct StarArgs {
   uint32_t table_len[TP_MAX_COLS], stride[TP_MAX_COLS];
   int agg;
   uint32_t ngroups;
+  uint32_t ht_slots, ht_shift;  // shared-memory aggregation table (grouped queries)
   long long* sums;
   unsigned long long* counts;
 };
 
-constexpr uint32_t HT_SLOTS = 2048, HT_EMPTY = 0xffffffffu, HT_PROBES = 64;
-constexpr uint32_t HT_WORDS = HT_SLOTS * 4;  // keys + sum lo + sum hi + counts, one word each per slot
+constexpr uint32_t HT_MAX_SLOTS = 2048, HT_EMPTY = 0xffffffffu, HT_PROBES = 64;
+// slots: a power of two >= 2 x the dense group count (at most 2048); 4 words per slot:
+// key, sum lo, sum hi, count
+static inline uint32_t ht_slots(uint32_t ngroups) {
+  uint32_t s = 256;
+  while (s < HT_MAX_SLOTS && s < 2u * ngroups) s <<= 1;
+  return s;
+}
 
 template <uint32_t MASK, bool GROUPED>
 struct StarOp : OpBase {
@@ -558,10 +616,10 @@ struct StarOp : OpBase {
   __device__ void cta_init(const Params& P, uint32_t* smem) {
     if (GROUPED) {
       keys = smem + P.agg_off;
-      hlo = keys + HT_SLOTS;
-      hhi = keys + 2 * HT_SLOTS;
-      hcnt = keys + 3 * HT_SLOTS;
-      for (uint32_t i = threadIdx.x; i < HT_SLOTS; i += blockDim.x) {
+      hlo = keys + A->ht_slots;
+      hhi = keys + 2 * A->ht_slots;
+      hcnt = keys + 3 * A->ht_slots;
+      for (uint32_t i = threadIdx.x; i < A->ht_slots; i += blockDim.x) {
         keys[i] = HT_EMPTY;
         hlo[i] = 0u;
         hhi[i] = 0u;
@@ -570,7 +628,7 @@ struct StarOp : OpBase {
     }
   }
   __device__ __forceinline__ void add(uint32_t key, int64_t v, uint32_t k) {
-    uint32_t slot = (key * 0x9E3779B1u) >> 21;  // 11-bit multiplicative hash
+    uint32_t slot = (key * 0x9E3779B1u) >> A->ht_shift;  // multiplicative hash
 #pragma unroll 1
     for (uint32_t p = 0; p < HT_PROBES; ++p) {
       uint32_t cur = keys[slot];
@@ -586,7 +644,7 @@ struct StarOp : OpBase {
         if (k) atomicAdd(&hcnt[slot], k);
         return;
       }
-      slot = (slot + 1u) & (HT_SLOTS - 1u);
+      slot = (slot + 1u) & (A->ht_slots - 1u);
     }
     atomicAdd(reinterpret_cast<unsigned long long*>(A->sums) + key, (unsigned long long)v);  // table crowded
     if (k) atomicAdd(A->counts + key, (unsigned long long)k);
@@ -663,7 +721,7 @@ struct StarOp : OpBase {
   __device__ void finish(const Params&, const Lane& g, uint32_t*) {
     if (GROUPED) {
       consumers_sync();
-      for (uint32_t i = threadIdx.x - 32u; i < HT_SLOTS; i += CONSUMER_WARPS * 32u) {
+      for (uint32_t i = threadIdx.x - 32u; i < A->ht_slots; i += CONSUMER_WARPS * 32u) {
         const uint32_t k = keys[i];
         if (k != HT_EMPTY) {
           atomicAdd(reinterpret_cast<unsigned long long*>(A->sums) + k,
@@ -784,6 +842,9 @@ static int sm_count() {
 #ifndef TP_RING_KB
 #define TP_RING_KB 40
 #endif
+#ifndef TP_QUERY_RING_KB
+#define TP_QUERY_RING_KB 24
+#endif
 static uint32_t worst_tile_words(uint32_t scheme) {
   return scheme == TP_FOR ? 4u * (2u + 128u) : scheme == TP_DFOR ? 1u + 4u * (2u + 128u) : 6u + 512u;
 }
@@ -865,7 +926,9 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
   // ring depth: 2..8 items within ~40 KB, so that several CTAs (16+ consumer warps) share
   // an SM while ~100+ KB of TMA traffic stays in flight per SM
   uint32_t nstg = TP_MAX_STAGES;
-  while (nstg > 2 && (size_t)nstg * P.stage_words * 4 > TP_RING_KB * 1024) --nstg;
+  // queries hold more per-warp state (3 CTAs/SM at most): a smaller ring keeps them at 3
+  const uint32_t ring_kb = ncols > 1 ? TP_QUERY_RING_KB : TP_RING_KB;
+  while (nstg > 2 && (size_t)nstg * P.stage_words * 4 > ring_kb * 1024) --nstg;
   P.nstages = nstg;
   P.scratch_off = nstg * P.stage_words;
   P.agg_off = P.scratch_off + CONSUMER_WARPS * P.scratch_words_per_warp;
@@ -1060,7 +1123,8 @@ tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int nc
   const bool grouped = ngroups > 1;
   Params P;
   size_t smem = 0;
-  tp_status st = build_params(dcols, ncols, 0, grouped ? HT_WORDS : 0u, P, smem);
+  const uint32_t hts = grouped ? ht_slots(ngroups) : 0u;
+  tp_status st = build_params(dcols, ncols, 0, 4u * hts, P, smem);
   if (st != TP_OK) return st;
   StarArgs A;
   memset(&A, 0, sizeof(A));
@@ -1071,6 +1135,8 @@ tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int nc
   }
   A.agg = agg;
   A.ngroups = ngroups;
+  A.ht_slots = hts;
+  A.ht_shift = 32u - (uint32_t)__builtin_ctz(hts ? hts : 1u);
   A.sums = reinterpret_cast<long long*>(d_sums);
   A.counts = reinterpret_cast<unsigned long long*>(d_counts);
   const int cap = (int)((P.ntiles + 1) / 2);
