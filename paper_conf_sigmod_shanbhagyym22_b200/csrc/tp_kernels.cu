@@ -78,6 +78,11 @@ __device__ __forceinline__ MbView for_mb(const Params& P, const Col& c, const St
 
 // ---------------------------------------------------------------- GPU-FOR decode
 // LoadBitPack analogue: the thread's 32 rows of the tile.
+// COMPACT: multi-column query kernels unpack with the runtime-bitwidth routine (one small
+// loop body instead of 33 specialised ones): their columns use several bitwidths at once, and
+// the specialised bodies thrash the instruction cache (measured: 24-34 % "no instruction"
+// stalls in the SSB kernel)
+template <bool COMPACT>
 __device__ __forceinline__ void decode_for(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                            uint32_t (&val)[32]) {
   const StreamView v = stream_view(P, c.s0, C);
@@ -85,7 +90,7 @@ __device__ __forceinline__ void decode_for(const Params& P, const Col& c, const 
   bool tv;
   const MbView m = for_mb(P, c, C, g, v, tl, tv);
   uint32_t e[32];
-  unpack_mb(m.w, m.b, e);
+  if (COMPACT) unpack_any(m.w, m.b, e); else unpack_mb(m.w, m.b, e);
 #pragma unroll
   for (int i = 0; i < 32; ++i) val[i] = m.ref + e[i];  // Alg. 1 line 18
 }
@@ -95,6 +100,7 @@ __device__ __forceinline__ void decode_for(const Params& P, const Col& c, const 
 // slots, then the tile-wide exclusive prefix sum (R13) -- a
 // register scan inside the thread plus a 16-lane shuffle scan across the
 // tile's miniblocks -- plus the tile's first value (Fig. 6).
+template <bool COMPACT>
 __device__ __forceinline__ void decode_dfor(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                             uint32_t (&val)[32]) {
   const StreamView v = stream_view(P, c.s0, C);
@@ -104,7 +110,7 @@ __device__ __forceinline__ void decode_dfor(const Params& P, const Col& c, const
   uint32_t first = 0u;
   if (tv) first = v.sd[v.ss[v.sshift + 4u * tl] - 1u - v.lo + v.dshift];
   uint32_t e[32];
-  unpack_mb(m.w, m.b, e);
+  if (COMPACT) unpack_any(m.w, m.b, e); else unpack_mb(m.w, m.b, e);
   uint32_t run = 0u;
 #pragma unroll
   for (int i = 0; i < 32; ++i) {  // local exclusive prefix of the deltas
@@ -248,12 +254,12 @@ __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const
 // MASK: which decoders a kernel instantiation carries (bit 1 << scheme); kernels
 // are instantiated per scheme mix so that FOR-only kernels keep FOR's register budget.
 constexpr uint32_t M_FOR = 1u << S_FOR, M_DFOR = 1u << S_DFOR, M_RFOR = 1u << S_RFOR;
-template <uint32_t MASK>
+template <uint32_t MASK, bool COMPACT = false>
 __device__ __forceinline__ void decode_col(const Params& P, uint32_t ci, const StageCtx& C, const Lane& g,
                                            uint32_t* scratch, uint32_t (&val)[32]) {
   const Col& c = P.col[ci];
-  if ((MASK & M_FOR) && c.scheme == S_FOR) decode_for(P, c, C, g, val);
-  else if ((MASK & M_DFOR) && c.scheme == S_DFOR) decode_dfor(P, c, C, g, val);
+  if ((MASK & M_FOR) && c.scheme == S_FOR) decode_for<COMPACT>(P, c, C, g, val);
+  else if ((MASK & M_DFOR) && c.scheme == S_DFOR) decode_dfor<COMPACT>(P, c, C, g, val);
   else if (MASK & M_RFOR) decode_rfor(P, c, C, g, scratch, val);
 }
 
@@ -310,7 +316,7 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
       for (uint32_t g = gb; g < ge; ++g) {
         const uint32_t tile_base = t0 + g * TPS, tile_end = min(tile_base + TPS, t1);
         for (uint32_t c = 0; c < P.ncols; ++c, ++item) {
-          if (item >= P.nstages) mbar_wait_backoff(&empty[slot], phase ^ 1u);
+          if (item >= P.nstages) mbar_wait(&empty[slot], phase ^ 1u);  // spin: fastest reaction (measured)
           const Col& cc = P.col[c];
           const uint32_t my_s = lane == 0 ? cc.s0 : (lane == 1 && cc.scheme == S_RFOR ? cc.s1 : 0xffu);
           uint32_t mylo = 0u, myhi = 0u;
@@ -404,6 +410,10 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
 __device__ __forceinline__ void consumers_sync() {
   asm volatile("bar.sync 1, %0;" ::"n"(CONSUMER_WARPS * 32) : "memory");
 }
+
+#ifndef TP_QUERY_COMPACT
+#define TP_QUERY_COMPACT true
+#endif
 
 // ------------------------------------------------------------------ consumers
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t x) {
@@ -540,7 +550,7 @@ struct SelectOp : OpBase {
   __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c, uint32_t) {
     if (!__any_sync(FULL, alive != 0u)) return;  // nothing survives in this warp's rows
     uint32_t v[32];
-    decode_col<MASK>(P, c, C, g, scratch, v);
+    decode_col<MASK, TP_QUERY_COMPACT>(P, c, C, g, scratch, v);
     const int32_t l = A->lo[c], h = A->hi[c];
 #pragma unroll
     for (int i = 0; i < 32; ++i)
@@ -627,7 +637,9 @@ struct StarOp : OpBase {
       }
     }
   }
-  __device__ __forceinline__ void add(uint32_t key, int64_t v, uint32_t k) {
+  // not inlined: the caller's 32-way unrolled row loop would otherwise carry 32 copies of the
+  // probe loop and its atomics (40 % of the kernel's code, an instruction-cache thrash)
+  __device__ __noinline__ void add(uint32_t key, int64_t v, uint32_t k) {
     uint32_t slot = (key * 0x9E3779B1u) >> A->ht_shift;  // multiplicative hash
 #pragma unroll 1
     for (uint32_t p = 0; p < HT_PROBES; ++p) {
@@ -664,7 +676,7 @@ struct StarOp : OpBase {
       return;
     }
     uint32_t v[32];
-    decode_col<MASK>(P, c, C, g, scratch, v);
+    decode_col<MASK, TP_QUERY_COMPACT>(P, c, C, g, scratch, v);
     if (role == TP_ROLE_PROBE) {
       const int32_t* __restrict__ T = A->table[c];
       const uint32_t kmin = (uint32_t)A->key_min[c], len = A->table_len[c], stride = A->stride[c];

@@ -53,7 +53,9 @@ def main():
     oracle = None
     if args.check and rank == 0:
         from oracle import ssb as ossb
+        t_o = time.perf_counter()
         oracle = ossb.SSB(db)
+        oracle_join_s = time.perf_counter() - t_o  # date join shared by all queries
     qs = QUERIES if args.queries == "all" else args.queries.split(",")
     res = {}
     for qid in qs:
@@ -100,11 +102,17 @@ def main():
             rows = eng.result(qid, prep, sums, counts)
             r["result_groups"] = len(rows)
             if oracle is not None:
-                r["parity"] = rows == oracle.run(qid)
+                t_o = time.perf_counter()
+                want = oracle.run(qid)
+                r["oracle_s"] = time.perf_counter() - t_o  # numpy SQL over uncompressed columns, host
+                r["parity"] = rows == want
             print(qid, json.dumps({k: (round(v, 4) if isinstance(v, float) else v) for k, v in r.items()}), flush=True)
         res[qid] = r
     if rank == 0:
         summary = {"sf": args.sf, "rows": n, "n_gpus": world, "gen_s": gen_s, "setup_s": setup_s,
+                   "cpu_baseline": None if oracle is None else {
+                       "kind": "oracle", "cores": 1, "what": "oracle/ssb.py: numpy SQL over the uncompressed "
+                       "columns, per query (oracle_s), plus a shared date join of %.2f s" % oracle_join_s},
                    "footprint": {k: [s, b] for k, (s, b) in eng.footprint().items()},
                    "geomean_query_ms": float(np.exp(np.mean([np.log(r["query_ms"]) for r in res.values()]))),
                    "queries": res}
