@@ -173,72 +173,72 @@ __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const
                                             uint32_t* scratch, uint32_t (&val)[32]) {
   const StreamView vv = stream_view(P, c.s0, C), vl = stream_view(P, c.s1, C);
   const uint32_t lane = g.lane;
-#pragma unroll 1
-  for (uint32_t h = 0; h < 2; ++h) {
-    uint32_t* bitmap = scratch + h * RFOR_HALF_WORDS;
-    uint32_t* V = bitmap + 16;
-    const uint32_t tl = C.round_base + 2u * g.cw + h;
-    const bool tv = C.t0s + tl < C.tile_end;
-    if (lane < 16) bitmap[lane] = 0u;
-    __syncwarp();
-    if (!tv) continue;  // warp-uniform
-    const uint32_t* bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
-    const uint32_t* bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
-    const uint32_t r = min(bV[0], 512u);  // run / value count
-    const uint32_t refV = bV[1], refL = bL[1];  // references (FOR on both arrays)
-    // 4 bitwidth words per stream: byte m = miniblock m (R2, R17)
-    const uint4 wv = make_uint4(bV[2], bV[3], bV[4], bV[5]);  // 4-byte aligned only: scalar loads
-    const uint4 wl = make_uint4(bL[2], bL[3], bL[4], bL[5]);
-    uint32_t carry = 0u;
-    // lane l takes entries 128q + 4l .. 128q + 4l + 3 of both streams: all four sit in
-    // miniblock 4q + l/8 (one bitwidth, and all earlier miniblocks are full, R17)
-    for (uint32_t q = 0; 128u * q < r; ++q) {
-      const uint32_t m = 4u * q + (lane >> 3);
-      const uint32_t e0 = 128u * q + 4u * lane;
-      const uint32_t bv = min(byte_of(wv, m), 32u), bl = min(byte_of(wl, m), 32u);
-      const uint32_t mv = __funnelshift_lc(0xffffffffu, 0u, bv), ml = __funnelshift_lc(0xffffffffu, 0u, bl);
-      const uint32_t* mV = bV + 6 + bytes_before(wv, m);  // miniblock m's first word
-      const uint32_t* mL = bL + 6 + bytes_before(wl, m);
-      const uint32_t pos = 4u * (lane & 7u);
-      uint32_t xv[4], len[4], incl[4];
-      uint32_t run = 0u;
+  // the warp's two row blocks are decoded side by side: half h = lane / 16 takes row block
+  // 2w + h, and lane t = lane % 16 of a half takes entries 128q + 8t .. 8t + 7 of both streams
+  const uint32_t h = lane >> 4, t = lane & 15u, hb = lane & 16u;
+  uint32_t* bitmap = scratch + h * RFOR_HALF_WORDS;
+  uint32_t* V = bitmap + 16;
+  const uint32_t tl = C.round_base + 2u * g.cw + h;
+  const bool tv = C.t0s + tl < C.tile_end;
+  bitmap[t] = 0u;
+  const uint32_t* bV = vv.sd;
+  const uint32_t* bL = vl.sd;
+  uint32_t r = 0u, refV = 0u, refL = 0u, bvt = 0u, blt = 0u;
+  if (tv) {
+    bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
+    bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
+    r = min(bV[0], 512u);  // run / value count
+    refV = bV[1];          // references (FOR on both arrays)
+    refL = bL[1];
+    // bitwidth byte t = miniblock t (R2, R17)
+    bvt = min((bV[2 + (t >> 2)] >> (8u * (t & 3u))) & 255u, 32u);
+    blt = min((bL[2 + (t >> 2)] >> (8u * (t & 3u))) & 255u, 32u);
+  }
+  // word offset of miniblock t: every earlier miniblock is full (b_i words), R17
+  const uint32_t offv = seg16_inclusive_scan(bvt) - bvt, offl = seg16_inclusive_scan(blt) - blt;
+  __syncwarp();
+  const uint32_t rmax = max(r, __shfl_xor_sync(FULL, r, 16));
+  uint32_t carry = 0u;
+  for (uint32_t q = 0; 128u * q < rmax; ++q) {
+    const uint32_t m = 4u * q + (t >> 2);  // miniblock of this lane's 8 entries
+    const uint32_t bv = __shfl_sync(FULL, bvt, hb + m), bl = __shfl_sync(FULL, blt, hb + m);
+    const uint32_t* mV = bV + 6 + __shfl_sync(FULL, offv, hb + m);
+    const uint32_t* mL = bL + 6 + __shfl_sync(FULL, offl, hb + m);
+    const uint32_t mv = __funnelshift_lc(0xffffffffu, 0u, bv), ml = __funnelshift_lc(0xffffffffu, 0u, bl);
+    const uint32_t e0 = 128u * q + 8u * t, pos = 8u * (t & 3u);
+    uint32_t len[8], incl[8];
+    uint32_t run = 0u;
 #pragma unroll
-      for (int k = 0; k < 4; ++k) {  // 1. unpack + local inclusive scan of the lengths
-        const bool in = e0 + k < r;
-        xv[k] = refV + extract_at(mV, (pos + k) * bv, mv);
-        len[k] = in ? refL + extract_at(mL, (pos + k) * bl, ml) : 0u;
-        run += len[k];
-        incl[k] = run;
-      }
-      // 2. warp scan of the per-lane totals -> run start rows
-      const uint32_t wincl = warp_inclusive_scan(run, lane);
-      const uint32_t base = carry + wincl - run;
-      // 3. scatter values and run-start bits (the 4 starts of a lane share at most a few words)
-      uint32_t cw = 0xffffffffu, cb = 0u;
-#pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        if (e0 + k < r) {
-          const uint32_t S = base + incl[k] - len[k];
-          V[e0 + k] = xv[k];
-          const uint32_t w = (S >> 5) & 15u;
-          if (w != cw) {
-            if (cb) atomicOr(&bitmap[cw], cb);
-            cw = w;
-            cb = 0u;
-          }
-          cb |= 1u << (S & 31u);
-        }
-      }
-      if (cb) atomicOr(&bitmap[cw], cb);
-      carry += __shfl_sync(FULL, wincl, 31);
+    for (int k = 0; k < 8; ++k) {  // 1. unpack the run lengths + local inclusive scan
+      len[k] = e0 + k < r ? refL + extract_at(mL, (pos + k) * bl, ml) : 0u;
+      run += len[k];
+      incl[k] = run;
     }
+    // 2. 16-lane scan of the per-lane totals -> run start rows
+    const uint32_t sincl = seg16_inclusive_scan(run);
+    const uint32_t base = carry + sincl - run;
+    // 3. values to smem, run-start bits to the bitmap (a lane's 8 starts span few words)
+    uint32_t cw = 0xffffffffu, cb = 0u;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      if (e0 + k < r) {
+        V[e0 + k] = refV + extract_at(mV, (pos + k) * bv, mv);
+        const uint32_t S = base + incl[k] - len[k];
+        const uint32_t w = (S >> 5) & 15u;
+        if (w != cw) {
+          if (cb) atomicOr(&bitmap[cw], cb);
+          cw = w;
+          cb = 0u;
+        }
+        cb |= 1u << (S & 31u);
+      }
+    }
+    if (cb) atomicOr(&bitmap[cw], cb);
+    carry += __shfl_sync(FULL, sincl, hb + 15u);
   }
   __syncwarp();
-  // 4. expand: rows 32j .. 32j+31 of row block h
-  const uint32_t h = lane >> 4, j = lane & 15u;
-  const uint32_t* bitmap = scratch + h * RFOR_HALF_WORDS;
-  const uint32_t* V = bitmap + 16;
-  const uint32_t bm = bitmap[j];
+  // 4. expand: rows 32t .. 32t+31 of row block h
+  const uint32_t bm = bitmap[t];
   const uint32_t pc = __popc(bm);
   const int before = (int)(seg16_inclusive_scan(pc) - pc);  // run starts before row 32j
 #pragma unroll
@@ -316,7 +316,12 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
       for (uint32_t g = gb; g < ge; ++g) {
         const uint32_t tile_base = t0 + g * TPS, tile_end = min(tile_base + TPS, t1);
         for (uint32_t c = 0; c < P.ncols; ++c, ++item) {
-          if (item >= P.nstages) mbar_wait(&empty[slot], phase ^ 1u);  // spin: fastest reaction (measured)
+          // HBM-bound single-column FOR decode: spin (fastest reaction, measured); everything
+          // else is consumer-bound: back off so the spin does not take the consumers' issue slots
+          if (item >= P.nstages) {
+            if (Op::kProducerSpin) mbar_wait(&empty[slot], phase ^ 1u);
+            else mbar_wait_backoff(&empty[slot], phase ^ 1u);
+          }
           const Col& cc = P.col[c];
           const uint32_t my_s = lane == 0 ? cc.s0 : (lane == 1 && cc.scheme == S_RFOR ? cc.s1 : 0xffu);
           uint32_t mylo = 0u, myhi = 0u;
@@ -431,6 +436,7 @@ __device__ __forceinline__ uint32_t valid_rows(const Params& P, const StageCtx& 
 }
 
 struct OpBase {
+  static constexpr bool kProducerSpin = false;
   __device__ void cta_init(const Params&, uint32_t*) {}
   __device__ void begin(const Params&, const StageCtx&, const Lane&) {}
   __device__ void end(const Params&, const StageCtx&, const Lane&) {}
@@ -439,6 +445,7 @@ struct OpBase {
 // decode -> sum (decode-only microbenchmark)
 template <uint32_t MASK>
 struct SumOp : OpBase {
+  static constexpr bool kProducerSpin = MASK == M_FOR;
   unsigned long long* out;
   uint64_t acc;
   __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t, uint32_t) {
@@ -490,6 +497,7 @@ struct SumOp : OpBase {
 // one TMA tensor store; the partial last miniblock (n % 32 rows) is stored directly.
 template <uint32_t MASK>
 struct GlobalOp : OpBase {
+  static constexpr bool kProducerSpin = true;  // HBM-bound (decoded rows are written back)
   const CUtensorMap* tmap;
   int32_t* out;
   uint32_t full_rows32;  // n / 32: rows of the [n/32][32] tensor
@@ -939,7 +947,10 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
   // an SM while ~100+ KB of TMA traffic stays in flight per SM
   uint32_t nstg = TP_MAX_STAGES;
   // queries hold more per-warp state (3 CTAs/SM at most): a smaller ring keeps them at 3
-  const uint32_t ring_kb = ncols > 1 ? TP_QUERY_RING_KB : TP_RING_KB;
+  // (FOR-only single columns are HBM-bound and get the big ring; DFOR / RFOR decodes are
+  // instruction-bound and trade ring space for one more resident CTA)
+  const bool for_only = ncols == 1 && P.col[0].scheme == S_FOR;
+  const uint32_t ring_kb = ncols > 1 ? TP_QUERY_RING_KB : (for_only ? TP_RING_KB : TP_QUERY_RING_KB);
   while (nstg > 2 && (size_t)nstg * P.stage_words * 4 > ring_kb * 1024) --nstg;
   P.nstages = nstg;
   P.scratch_off = nstg * P.stage_words;
