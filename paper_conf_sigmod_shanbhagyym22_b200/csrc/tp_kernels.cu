@@ -217,23 +217,15 @@ __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const
     // 2. 16-lane scan of the per-lane totals -> run start rows
     const uint32_t sincl = seg16_inclusive_scan(run);
     const uint32_t base = carry + sincl - run;
-    // 3. values to smem, run-start bits to the bitmap (a lane's 8 starts span few words)
-    uint32_t cw = 0xffffffffu, cb = 0u;
+    // 3. values to smem, run-start bits to the bitmap (predicated, branch-free)
 #pragma unroll
     for (int k = 0; k < 8; ++k) {
+      const uint32_t S = base + incl[k] - len[k];
       if (e0 + k < r) {
         V[e0 + k] = refV + extract_at(mV, (pos + k) * bv, mv);
-        const uint32_t S = base + incl[k] - len[k];
-        const uint32_t w = (S >> 5) & 15u;
-        if (w != cw) {
-          if (cb) atomicOr(&bitmap[cw], cb);
-          cw = w;
-          cb = 0u;
-        }
-        cb |= 1u << (S & 31u);
+        atomicOr(&bitmap[(S >> 5) & 15u], 1u << (S & 31u));
       }
     }
-    if (cb) atomicOr(&bitmap[cw], cb);
     carry += __shfl_sync(FULL, sincl, hb + 15u);
   }
   __syncwarp();
