@@ -54,11 +54,14 @@ def date_dim() -> dict:
             "d_weeknuminyear": a(week)}
 
 
-def generate(sf: float, seed: int = 5000) -> dict:
-    """Returns {'lineorder': {col: int32 array}, 'date': ..., 'customer': ..., 'supplier': ..., 'part': ...}."""
+def generate(sf: float, seed: int = 5000, columns=None) -> dict:
+    """Returns {'lineorder': {col: int32 array}, 'date': ..., 'customer': ..., 'supplier': ..., 'part': ...}.
+    `columns` restricts the lineorder columns returned (same values either way: every random
+    stream is drawn in the same order)."""
     rng = np.random.default_rng(seed)
     z = sizes(sf)
     C, S, P, O = z["customer"], z["supplier"], z["part"], z["orders"]
+    want = set(columns) if columns is not None else set(LINEORDER_COLUMNS)
     date = date_dim()
     # dimensions (keys are dense 1..N; attributes uniform like dbgen)
     c_nation = rng.integers(0, 25, C, dtype=np.int32)
@@ -71,7 +74,7 @@ def generate(sf: float, seed: int = 5000) -> dict:
     cat = mfgr * 10 + rng.integers(1, 6, P, dtype=np.int32)
     brand = cat * 100 + rng.integers(1, 41, P, dtype=np.int32)
     pk = np.arange(1, P + 1, dtype=np.int64)
-    retail = (90000 + (pk // 10) % 20001 + 100 * (pk % 1000)).astype(np.int64)  # TPC-H p_retailprice (cents)
+    retail = (90000 + (pk // 10) % 20001 + 100 * (pk % 1000)).astype(np.int32)  # TPC-H p_retailprice (cents)
     part = {"p_partkey": pk.astype(np.int32), "p_mfgr": mfgr, "p_category": cat, "p_brand1": brand}
     # orders: 1..7 lines, date in [1992-01-01, 1998-08-02], custkey, priority constant per order
     lines = rng.integers(1, 8, O, dtype=np.int64)
@@ -83,28 +86,36 @@ def generate(sf: float, seed: int = 5000) -> dict:
     ocust = rng.integers(1, C + 1, O, dtype=np.int32)
     oprio = rng.integers(1, 6, O, dtype=np.int32)
     rep = lambda v: np.repeat(v, lines)  # noqa: E731
-    lo_orderkey = rep(okey).astype(np.int32)
-    starts = np.cumsum(lines) - lines
-    lo_linenumber = (np.arange(n, dtype=np.int64) - rep(starts) + 1).astype(np.int32)
-    qty = rng.integers(1, 51, n, dtype=np.int64)
-    disc = rng.integers(0, 11, n, dtype=np.int64)
-    tax = rng.integers(0, 9, n, dtype=np.int64)
-    lo_partkey = rng.integers(1, P + 1, n, dtype=np.int64)
+    lo = {}
+    if "lo_orderkey" in want:
+        lo["lo_orderkey"] = rep(okey).astype(np.int32)
+    if "lo_linenumber" in want:
+        starts = np.cumsum(lines) - lines
+        lo["lo_linenumber"] = (np.arange(n, dtype=np.int64) - rep(starts) + 1).astype(np.int32)
+    qty = rng.integers(1, 51, n, dtype=np.int32)
+    disc = rng.integers(0, 11, n, dtype=np.int32)
+    tax = rng.integers(0, 9, n, dtype=np.int32)
+    lo_partkey = rng.integers(1, P + 1, n, dtype=np.int32)
     lo_suppkey = rng.integers(1, S + 1, n, dtype=np.int32)
-    ext = qty * retail[lo_partkey - 1]
-    rev = ext * (100 - disc) // 100
-    supplycost = rng.integers(100, 100_001, n, dtype=np.int64)
-    otot = np.bincount(np.repeat(np.arange(O), lines), weights=rev, minlength=O).astype(np.int64)
+    ext = qty * retail[lo_partkey - 1]                      # < 50 * 2.1e6: fits int32
+    rev = (ext.astype(np.int64) * (100 - disc) // 100).astype(np.int32)
+    supplycost = rng.integers(100, 100_001, n, dtype=np.int32)
+    if "lo_ordtotalprice" in want:
+        otot = np.bincount(np.repeat(np.arange(O), lines), weights=rev, minlength=O).astype(np.int64)
+        lo["lo_ordtotalprice"] = np.minimum(rep(otot), 2**31 - 1).astype(np.int32)
     lo_orderdate = rep(odate).astype(np.int32)
-    dayidx = np.searchsorted(date["d_datekey"], lo_orderdate)
-    commit = date["d_datekey"][np.minimum(dayidx + rng.integers(30, 91, n), len(date["d_datekey"]) - 1)]
-    lineorder = {
-        "lo_orderkey": lo_orderkey, "lo_linenumber": lo_linenumber, "lo_custkey": rep(ocust).astype(np.int32),
-        "lo_partkey": lo_partkey.astype(np.int32), "lo_suppkey": lo_suppkey, "lo_orderdate": lo_orderdate,
-        "lo_orderpriority": rep(oprio).astype(np.int32), "lo_quantity": qty.astype(np.int32),
-        "lo_extendedprice": ext.astype(np.int32), "lo_ordtotalprice": np.minimum(rep(otot), 2**31 - 1).astype(np.int32),
-        "lo_discount": disc.astype(np.int32), "lo_revenue": rev.astype(np.int32),
-        "lo_supplycost": supplycost.astype(np.int32), "lo_tax": tax.astype(np.int32),
-        "lo_commitdate": commit.astype(np.int32)}
+    if "lo_commitdate" in want:
+        dayidx = np.searchsorted(date["d_datekey"], lo_orderdate)
+        lo["lo_commitdate"] = date["d_datekey"][np.minimum(dayidx + rng.integers(30, 91, n),
+                                                           len(date["d_datekey"]) - 1)].astype(np.int32)
+    full = {"lo_custkey": lambda: rep(ocust).astype(np.int32), "lo_partkey": lambda: lo_partkey,
+            "lo_suppkey": lambda: lo_suppkey, "lo_orderdate": lambda: lo_orderdate,
+            "lo_orderpriority": lambda: rep(oprio).astype(np.int32), "lo_quantity": lambda: qty,
+            "lo_extendedprice": lambda: ext, "lo_discount": lambda: disc, "lo_revenue": lambda: rev,
+            "lo_supplycost": lambda: supplycost, "lo_tax": lambda: tax}
+    for k, f in full.items():
+        if k in want:
+            lo[k] = f()
+    lineorder = {k: lo[k] for k in LINEORDER_COLUMNS if k in lo}
     return {"sf": sf, "lineorder": lineorder, "date": date, "customer": customer, "supplier": supplier,
             "part": part}

@@ -40,7 +40,7 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
     t0 = time.time()
-    db = gen.generate(args.sf, seed=5000)
+    db = gen.generate(args.sf, seed=5000, columns=gen.QUERY_COLUMNS)
     n = len(db["lineorder"]["lo_orderdate"])
     from paper_conf_sigmod_shanbhagyym22_b200.dist import tile_range
     r0, r1 = tile_range(n, rank, world)
