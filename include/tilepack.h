@@ -202,6 +202,16 @@ tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int nc
  * Used as the measured HBM read roof of the same consumer. */
 tp_status tp_plain_sum(const int32_t* d_x, uint64_t n, int64_t* d_sum, void* stream);
 
+/* ------------------------------------------------ cascading baseline (ablation)
+ * The paper's CASCADING decompression model, the baseline of
+ * Fig. 7a: the same encoded DEVICE column decoded one layer per kernel, every layer
+ * reading and writing global memory -- FOR+BitPack 2 passes, Delta+FOR+BitPack 3,
+ * RLE+FOR+BitPack 8.  d_out receives the n decoded values (as tp_decode); d_work is a
+ * DEVICE scratch of tp_cascaded_workspace_words(col) u32 words.  For measurement only
+ * (SURVEY.md NEXT-1). */
+uint64_t tp_cascaded_workspace_words(const tp_column* col);
+tp_status tp_decode_cascaded(const tp_column* dcol, int32_t* d_out, uint32_t* d_work, void* stream);
+
 /* --------------------------------------------------------------- utility */
 
 const char* tp_status_string(tp_status s);

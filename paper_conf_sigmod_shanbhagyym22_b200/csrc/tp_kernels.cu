@@ -82,7 +82,9 @@ __device__ __forceinline__ MbView for_mb(const Params& P, const Col& c, const St
 // loop body instead of 33 specialised ones): their columns use several bitwidths at once, and
 // the specialised bodies thrash the instruction cache (measured: 24-34 % "no instruction"
 // stalls in the SSB kernel)
-template <bool COMPACT>
+// RAW: the packed offsets only (no reference added) -- the first pass of the cascading
+// baseline (tp_cascaded.cu), also for the delta blocks of a GPU-DFOR column
+template <bool COMPACT, bool RAW = false>
 __device__ __forceinline__ void decode_for(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                            uint32_t (&val)[32]) {
   const StreamView v = stream_view(P, c.s0, C);
@@ -92,7 +94,7 @@ __device__ __forceinline__ void decode_for(const Params& P, const Col& c, const 
   uint32_t e[32];
   if (COMPACT) unpack_any(m.w, m.b, e); else unpack_mb(m.w, m.b, e);
 #pragma unroll
-  for (int i = 0; i < 32; ++i) val[i] = m.ref + e[i];  // Alg. 1 line 18
+  for (int i = 0; i < 32; ++i) val[i] = RAW ? e[i] : m.ref + e[i];  // Alg. 1 line 18
 }
 
 // ---------------------------------------------------------------- GPU-DFOR decode
@@ -246,10 +248,15 @@ __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const
 // MASK: which decoders a kernel instantiation carries (bit 1 << scheme); kernels
 // are instantiated per scheme mix so that FOR-only kernels keep FOR's register budget.
 constexpr uint32_t M_FOR = 1u << S_FOR, M_DFOR = 1u << S_DFOR, M_RFOR = 1u << S_RFOR;
+constexpr uint32_t M_RAW = 1u << 8;  // FOR / DFOR blocks, packed offsets only (cascading baseline)
 template <uint32_t MASK, bool COMPACT = false>
 __device__ __forceinline__ void decode_col(const Params& P, uint32_t ci, const StageCtx& C, const Lane& g,
                                            uint32_t* scratch, uint32_t (&val)[32]) {
   const Col& c = P.col[ci];
+  if (MASK == M_RAW) {
+    decode_for<false, true>(P, c, C, g, val);
+    return;
+  }
   if ((MASK & M_FOR) && c.scheme == S_FOR) decode_for<COMPACT>(P, c, C, g, val);
   else if ((MASK & M_DFOR) && c.scheme == S_DFOR) decode_dfor<COMPACT>(P, c, C, g, val);
   else if (MASK & M_RFOR) decode_rfor(P, c, C, g, scratch, val);
@@ -1026,10 +1033,15 @@ tp_status tp_decode_sum(const tp_column* dcol, int64_t* d_sum, void* stream) {
   return launched();
 }
 
-tp_status tp_decode(const tp_column* dcol, int32_t* d_out, void* stream) {
+}  // extern "C"
+
+namespace tp {
+// decode -> global through the tile pipeline; raw = packed offsets only (FOR / DFOR blocks)
+tp_status decode_global_impl(const tp_column* dcol, int32_t* d_out, bool raw, void* stream) {
   if (!dcol || !d_out) return TP_EINVAL;
   if (dcol->n == 0) return TP_OK;
   if (reinterpret_cast<uintptr_t>(d_out) & 15u) return TP_EINVAL;
+  if (raw && dcol->scheme == TP_RFOR) return TP_EINVAL;
   Params P;
   size_t smem = 0;
   // per warp: 2 x 4 KB swizzled staging + 1 KB alignment slop
@@ -1051,12 +1063,23 @@ tp_status tp_decode(const tp_column* dcol, int32_t* d_out, void* stream) {
       return TP_ECUDA;
   }
   const int cap = (int)((P.ntiles + 1) / 2);
+  if (raw) {
+    launch(k_decode_global<M_RAW>, smem, cap, stream, P, tmap, d_out);
+    return launched();
+  }
   switch (scheme_mask(P)) {
     case M_FOR: launch(k_decode_global<M_FOR>, smem, cap, stream, P, tmap, d_out); break;
     case M_DFOR: launch(k_decode_global<M_DFOR>, smem, cap, stream, P, tmap, d_out); break;
     default: launch(k_decode_global<M_RFOR>, smem, cap, stream, P, tmap, d_out); break;
   }
   return launched();
+}
+}  // namespace tp
+
+extern "C" {
+
+tp_status tp_decode(const tp_column* dcol, int32_t* d_out, void* stream) {
+  return decode_global_impl(dcol, d_out, false, stream);
 }
 
 tp_status tp_select_project_sum(const tp_column* dcols, int ncols, const int32_t* lo, const int32_t* hi, int proj_op,

@@ -79,6 +79,8 @@ def _load():
         "tp_decode_sum": (i32, [colp, vp, vp]),
         "tp_select_project_sum": (i32, [colp, i32, vp, vp, i32, i32, i32, vp, vp]),
         "tp_plain_sum": (i32, [vp, u64, vp, vp]),
+        "tp_cascaded_workspace_words": (u64, [colp]),
+        "tp_decode_cascaded": (i32, [colp, vp, vp, vp]),
         "tp_lookup_build": (i32, [vp, u64, ctypes.c_int32, u32, ctypes.POINTER(tp_dim_pred), i32, vp, vp, vp]),
         "tp_star_query": (i32, [colp, ctypes.POINTER(tp_star_col), i32, i32, vp, vp, u32, vp]),
         "tp_status_string": (ctypes.c_char_p, [i32]),
@@ -185,6 +187,27 @@ def tp_star_query(dcols, roles, agg: int, d_sums, d_counts, ngroups: int, stream
     rarr = (tp_star_col * n)(*roles)
     _check(_lib.tp_star_query(carr, rarr, n, agg, _ptr(d_sums), _ptr(d_counts), ngroups, _stream(stream)),
            "tp_star_query")
+
+
+def tp_cascaded_workspace_words(col: tp_column) -> int:
+    return int(_lib.tp_cascaded_workspace_words(ctypes.byref(col)))
+
+
+def tp_decode_cascaded(dcol: tp_column, d_out, d_work, stream=None):
+    _check(_lib.tp_decode_cascaded(ctypes.byref(dcol), _ptr(d_out), _ptr(d_work), _stream(stream)),
+           "tp_decode_cascaded")
+
+
+def decode_cascaded(dcol: "DeviceColumn", out=None, work=None, stream=None):
+    """The cascading-decompression baseline (one kernel per layer)."""
+    import torch
+    dev = dcol.data0.device
+    if out is None:
+        out = torch.empty(dcol.n, dtype=torch.int32, device=dev)
+    if work is None:
+        work = torch.empty(max(1, tp_cascaded_workspace_words(dcol.col)), dtype=torch.int32, device=dev)
+    tp_decode_cascaded(dcol.col, out, work, stream)
+    return out
 
 
 def tp_plain_sum(d_x, n: int, d_sum, stream=None):

@@ -145,3 +145,17 @@ def test_fake_multi_gpu_shards(scheme):
             tp.decode_sum(d, out=acc)
         assert np.array_equal(np.concatenate(pieces), x)
         assert int(acc.item()) == oracle.column_sum(x)
+
+
+@pytest.mark.parametrize("scheme", SCHEMES)
+def test_cascaded_baseline_parity(scheme):
+    """NEXT-1: the cascading-decompression baseline decodes the same bytes to the same values."""
+    for name, x in list(datagen.mixed_columns(seed=21))[::3]:
+        if len(x) == 0:
+            continue
+        d = tp.encode(x, scheme).to_device()
+        assert np.array_equal(tp.decode_cascaded(d).cpu().numpy(), x), (scheme, name)
+    x = {"for": datagen.uniform_bits(12, 3_000_001, seed=4), "dfor": datagen.near_sorted(3_000_001, seed=4),
+         "rfor": datagen.runs(3_000_001, 6, seed=4)}[scheme]
+    d = tp.encode(x, scheme).to_device()
+    assert np.array_equal(tp.decode_cascaded(d).cpu().numpy(), x)
