@@ -180,7 +180,14 @@ tp_status tp_lookup_build(const int32_t* d_keys, uint64_t nrows, int32_t key_min
  *                     [INT32_MIN, INT32_MAX] for none); agg (below) combines
  *                     the measures: TP_AGG_SUM: sum(m0); TP_AGG_MUL:
  *                     sum(m0 * m1); TP_AGG_SUB: sum(m0 - m1)  (int64, R24)
- * Put MEASURE columns last; with TP_AGG_SUB only m0 may carry a filter.  For every surviving row:
+ * The LAST column is the aggregating measure (m1 for MUL / SUB, m0 for SUM);
+ * with MUL / SUB exactly one earlier column is a MEASURE (m0), which may sit
+ * anywhere before it (its value is staged per row; filters after it still
+ * apply).  Columns are evaluated in the order given: put the most selective
+ * first -- once few rows of a warp survive, later columns are read row by row
+ * (random access into the staged tile) instead of decoded whole.
+ * Errors: TP_EINVAL for a bad role / missing table / measure layout.
+ * For every surviving row:
  *   d_sums[group] += aggregate, d_counts[group] += 1
  * (DEVICE int64 / uint64 arrays of ngroups, caller-zeroed).  Rows whose group
  * is >= ngroups are a caller error (not checked per row). */
@@ -219,6 +226,10 @@ const char* tp_status_string(tp_status s);
 /* Number of CUDA kernels this library has launched in this process
  * (bench.py reports it as gpu_launches). */
 uint64_t tp_launch_count(void);
+/* Profiling builds only (-DTP_PROFILE_WAITS): copy 16 cycle counters of the query pipeline
+ * (consumer data waits, per-column work, producer slot waits) to out16 (host) and reset
+ * them.  Other builds report zeros. */
+tp_status tp_debug_counters(uint64_t* out16);
 
 /* Number of SMs of the current device and the decoder's CTAs per SM
  * (persistent grid = SMs x CTAs/SM). */

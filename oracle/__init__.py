@@ -231,3 +231,42 @@ def select_project_sum(cols, lo, hi, proj: str = "col", a: int = 0, b: int = 0) 
 def column_sum(x) -> int:
     x = _col(x)
     return int(lib().orc_sum(_p(x), len(x)))
+
+
+def star_query(cols, roles, agg: str, ngroups: int):
+    """One star-join pass by its plain definition (include/tilepack.h tp_star_query; SSB
+    star joins P:1874-1888): rows survive every RANGE (lo <= v <= hi), every PROBE
+    (p = table[v - key_min] >= 0, group += p * stride) and every MEASURE's own range;
+    the last column is the aggregating measure m_last, an earlier measure is m_first;
+    aggregate = m_last (sum) | m_first * m_last (mul) | m_first - m_last (sub), int64.
+    roles: dicts {role: "range"|"probe"|"measure", lo, hi, table (np int32), key_min, stride}.
+    Returns (sums[ngroups] int64, counts[ngroups] int64).  Plain numpy, row-parallel."""
+    cols = [np.asarray(c, np.int64) for c in cols]
+    n = len(cols[0])
+    alive = np.ones(n, bool)
+    group = np.zeros(n, np.int64)
+    meas = []
+    for x, r in zip(cols, roles):
+        if r["role"] == "probe":
+            t = np.asarray(r["table"], np.int64)
+            k = x - r["key_min"]
+            inside = (k >= 0) & (k < len(t))
+            p = np.full(n, -1, np.int64)
+            p[inside] = t[k[inside]]
+            alive &= p >= 0
+            group += np.where(p >= 0, p, 0) * r.get("stride", 0)
+        else:
+            alive &= (x >= r["lo"]) & (x <= r["hi"])
+            if r["role"] == "measure":
+                meas.append(x)
+    if agg == "sum":
+        y = meas[-1]
+    elif agg == "mul":
+        y = meas[0] * meas[1]
+    else:
+        y = meas[0] - meas[1]
+    g = group[alive] if ngroups > 1 else np.zeros(int(alive.sum()), np.int64)
+    sums = np.zeros(ngroups, np.int64)
+    np.add.at(sums, g, y[alive])
+    counts = np.bincount(g, minlength=ngroups).astype(np.int64)
+    return sums, counts

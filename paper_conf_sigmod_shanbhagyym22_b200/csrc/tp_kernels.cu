@@ -10,6 +10,7 @@
 #include <algorithm>
 #include <atomic>
 #include <climits>
+#include <cstdlib>
 #include <cstring>
 
 #include "tilepack.h"
@@ -18,6 +19,9 @@
 namespace tp {
 
 std::atomic<uint64_t> g_launches{0};
+// TP_PROFILE_WAITS builds only: consumer full-wait cycles [0], per-column op cycles [1..7],
+// producer empty-wait cycles [8] (summed over warps)
+__device__ unsigned long long g_prof[16];
 
 // ------------------------------------------------------------------ stage context
 // The ring holds "items": one column's words for a range of TPR * rounds consecutive
@@ -126,16 +130,22 @@ __device__ __forceinline__ void decode_dfor(const Params& P, const Col& c, const
 }
 
 // ---------------------------------------------------------------- GPU-RFOR decode
-// LoadRBitPack analogue.  Per row block (a warp does 2 per round):
-//  1. lane-per-entry unpack of the value and run-length stream blocks, 32 entries
-//     (= one miniblock, warp-uniform bitwidth) per step;
-//  2. warp scan of the run lengths -> run start rows S (the first inclusive scan of [18]);
-//  3. scatter: value V_e -> smem, bit S_e -> a 512-bit run-start bitmap (the scatters of [18]);
-//  4. expand: the thread owning rows 32j..32j+31 counts run starts before its rows
-//     (popcount + 16-lane scan = the second scan of [18]) and walks its bitmap word.
-// The result equals repeat(V, L) (R19).
-constexpr uint32_t RFOR_HALF_WORDS = 16 + 512 + 32;  // bitmap + values + pad: the halves sit 16 banks apart
-constexpr uint32_t RFOR_SCRATCH_WORDS = 2 * RFOR_HALF_WORDS;
+// LoadRBitPack analogue: the 4 steps of [18] (2 scatters + 2 scans),
+// done per 512-row block by one warp, both blocks of the warp's round in turn:
+//  1. unpack: lane t takes the C consecutive entries [C t, C t + C) of both streams
+//     (C = 4 / 8 / 16 by the block's run count r, so one pass covers the block and a lane's
+//     entries sit inside one 32-entry miniblock: one bitwidth and base per lane);
+//  2. run starts S = exclusive scan of the run lengths (lane-local scan + one warp scan);
+//  3. scatter: value V_e -> A[S_e], a start flag byte -> F[S_e] (plain stores: the starts
+//     are distinct, no atomics);
+//  4. expand (second scan): the thread owning rows 32j .. 32j+31 turns its 32 flag bytes
+//     into a start mask, takes the value of the last run start before its rows from the
+//     nearest earlier thread (16-lane segmented scan), and forward-fills its rows.
+// A is stored XOR-swizzled by 16-byte quad so that the 16 threads' 128-bit reads of
+// their row chunks are conflict-free.  The result equals repeat(V, L) (R19).
+constexpr uint32_t RFOR_A_WORDS = 512, RFOR_F_WORDS = 128;
+constexpr uint32_t RFOR_BLOCK_WORDS = RFOR_A_WORDS + RFOR_F_WORDS;
+constexpr uint32_t RFOR_SCRATCH_WORDS = 2 * RFOR_BLOCK_WORDS;
 
 __device__ __forceinline__ uint32_t warp_inclusive_scan(uint32_t x, uint32_t lane) {
 #pragma unroll
@@ -144,13 +154,6 @@ __device__ __forceinline__ uint32_t warp_inclusive_scan(uint32_t x, uint32_t lan
     if (lane >= (uint32_t)d) x += y;
   }
   return x;
-}
-
-// entry `lane` of a b-bit miniblock at m (lane-per-entry); `mask` = 2^b - 1
-__device__ __forceinline__ uint32_t extract_lane(const uint32_t* m, uint32_t lane, uint32_t b, uint32_t mask) {
-  const uint32_t p = lane * b;
-  const uint32_t* w = m + (p >> 5);
-  return __funnelshift_r(w[0], w[1], p) & mask;  // the funnel shift uses p mod 32
 }
 
 __device__ __forceinline__ uint32_t byte_of(const uint4& w, uint32_t m) {  // byte m (0..15)
@@ -170,79 +173,124 @@ __device__ __forceinline__ uint32_t extract_at(const uint32_t* m, uint32_t p, ui
   const uint32_t* w = m + (p >> 5);
   return __funnelshift_r(w[0], w[1], p) & mask;
 }
+// swizzled word / flag-byte positions of row s of a block (see above)
+__device__ __forceinline__ uint32_t rfor_a_pos(uint32_t s) { return s ^ ((s >> 3) & 0x1Cu); }
+__device__ __forceinline__ uint32_t rfor_f_pos(uint32_t s) { return s ^ (((s >> 7) & 1u) << 4); }
+
+// steps 1-3 for one block, C entries per lane
+template <int C>
+__device__ __forceinline__ void rfor_scatter(const uint32_t* bV, const uint32_t* bL, uint32_t r, uint32_t lane,
+                                             uint32_t* A, uint8_t* F) {
+  const uint32_t e0 = C * lane, m = e0 >> 5, pos = e0 & 31u;
+  const uint32_t refV = bV[1], refL = bL[1];  // references (FOR on both arrays)
+  const uint4 wv = make_uint4(bV[2], bV[3], bV[4], bV[5]), wl = make_uint4(bL[2], bL[3], bL[4], bL[5]);
+  const uint32_t bv = min(byte_of(wv, m), 32u), bl = min(byte_of(wl, m), 32u);  // R2, R17
+  // every miniblock before m is full: b_i words each (R17)
+  const uint32_t* mV = bV + 6 + bytes_before(wv, m);
+  const uint32_t* mL = bL + 6 + bytes_before(wl, m);
+  const uint32_t mv = __funnelshift_lc(0xffffffffu, 0u, bv), ml = __funnelshift_lc(0xffffffffu, 0u, bl);
+  uint32_t len[C], incl[C];
+  uint32_t run = 0u;
+#pragma unroll
+  for (int k = 0; k < C; ++k) {  // 1. run lengths + lane-local inclusive scan
+    len[k] = e0 + k < r ? refL + extract_at(mL, (pos + k) * bl, ml) : 0u;
+    run += len[k];
+    incl[k] = run;
+  }
+  const uint32_t base = warp_inclusive_scan(run, lane) - run;  // 2. rows before this lane's runs
+#pragma unroll
+  for (int k = 0; k < C; ++k) {  // 3. scatter values and start flags
+    if (e0 + k < r) {
+      const uint32_t S = (base + incl[k] - len[k]) & 511u;
+      A[rfor_a_pos(S)] = refV + extract_at(mV, (pos + k) * bv, mv);
+      F[rfor_f_pos(S)] = 1;
+    }
+  }
+}
+
+// steps 1-3 for both row blocks of the warp's round (block h -> scratch + h * RFOR_BLOCK_WORDS)
+__device__ __forceinline__ void rfor_scatter_round(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
+                                                   uint32_t* scratch) {
+  const StreamView vv = stream_view(P, c.s0, C), vl = stream_view(P, c.s1, C);
+  const uint32_t lane = g.lane;
+  __syncwarp();  // a lagging lane may still read the previous column's expansion
+#pragma unroll 1
+  for (uint32_t h = 0; h < 2; ++h) {
+    uint32_t* A = scratch + h * RFOR_BLOCK_WORDS;
+    uint8_t* F = reinterpret_cast<uint8_t*>(A + RFOR_A_WORDS);
+    st_shared_v4(reinterpret_cast<uint32_t*>(F) + 4u * lane, 0u, 0u, 0u, 0u);
+    __syncwarp();
+    const uint32_t tl = C.round_base + 2u * g.cw + h;
+    if (C.t0s + tl >= C.tile_end) continue;  // warp-uniform; rows masked by the consumer
+    const uint32_t* bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
+    const uint32_t* bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
+    const uint32_t r = min(bV[0], 512u);  // run / value count
+    if (r <= 128u) rfor_scatter<4>(bV, bL, r, lane, A, F);
+    else if (r <= 256u) rfor_scatter<8>(bV, bL, r, lane, A, F);
+    else rfor_scatter<16>(bV, bL, r, lane, A, F);
+  }
+  __syncwarp();
+}
+
+// the thread's 32-row chunk of an expanded RFOR round: run-start mask and value array
+struct RforChunk {
+  uint32_t* A;    // the block's (swizzled) start-value array
+  uint32_t j;     // chunk index in the block (rows 32j .. 32j+31)
+  uint32_t mask;  // bit i: row 32j+i starts a run
+};
+__device__ __forceinline__ RforChunk rfor_chunk(uint32_t* scratch, uint32_t lane) {
+  RforChunk k;
+  k.j = lane & 15u;
+  k.A = scratch + (lane >> 4) * RFOR_BLOCK_WORDS;
+  const uint32_t* F = k.A + RFOR_A_WORDS;
+  const uint32_t fs = ((k.j >> 2) & 1u) << 2;  // flag quad swizzle (words)
+  const uint4 f0 = *reinterpret_cast<const uint4*>(F + 8u * k.j + fs);
+  const uint4 f1 = *reinterpret_cast<const uint4*>(F + 8u * k.j + (fs ^ 4u));
+  const uint32_t fw[8] = {f0.x, f0.y, f0.z, f0.w, f1.x, f1.y, f1.z, f1.w};
+  uint32_t mask = 0u;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) mask |= (((fw[q] * 0x01020408u) >> 24) & 15u) << (4 * q);  // byte flags -> bits
+  k.mask = mask;
+  return k;
+}
+// A-value of the last run start before row 32j (the previous chunks' last start: a 16-lane
+// segmented scan -- the second scan of [18]); row 0 of a block always starts a run
+__device__ __forceinline__ uint32_t rfor_carry(const RforChunk& k) {
+  uint32_t has = k.mask != 0u;
+  uint32_t last = has ? k.A[rfor_a_pos(32u * k.j + 31u - __clz(k.mask))] : 0u;
+#pragma unroll
+  for (int d = 1; d < 16; d <<= 1) {
+    const uint32_t yh = __shfl_up_sync(FULL, has, d, 16), yv = __shfl_up_sync(FULL, last, d, 16);
+    if (k.j >= (uint32_t)d && !has) { has = yh; last = yv; }
+  }
+  return __shfl_up_sync(FULL, last, 1, 16);
+}
+// step 4: forward fill of the chunk's 32 rows
+__device__ __forceinline__ void rfor_fill(const RforChunk& k, uint32_t carry, uint32_t (&val)[32]) {
+  const uint32_t* Aj = k.A + 32u * k.j;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const uint4 a = *reinterpret_cast<const uint4*>(Aj + ((q ^ (k.j & 7u)) << 2));
+    val[4 * q] = a.x; val[4 * q + 1] = a.y; val[4 * q + 2] = a.z; val[4 * q + 3] = a.w;
+  }
+  uint32_t cur = carry;
+#pragma unroll
+  for (int i = 0; i < 32; ++i) {
+    if (k.mask & (1u << i)) cur = val[i];
+    val[i] = cur;
+  }
+}
+// random access: the value of row 32j + i (the last run start at or before it)
+__device__ __forceinline__ uint32_t rfor_row(const RforChunk& k, uint32_t carry, uint32_t i) {
+  const uint32_t mm = k.mask & (0xffffffffu >> (31u - i));
+  return mm ? k.A[rfor_a_pos(32u * k.j + 31u - __clz(mm))] : carry;
+}
 
 __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                             uint32_t* scratch, uint32_t (&val)[32]) {
-  const StreamView vv = stream_view(P, c.s0, C), vl = stream_view(P, c.s1, C);
-  const uint32_t lane = g.lane;
-  // the warp's two row blocks are decoded side by side: half h = lane / 16 takes row block
-  // 2w + h, and lane t = lane % 16 of a half takes entries 128q + 8t .. 8t + 7 of both streams
-  const uint32_t h = lane >> 4, t = lane & 15u, hb = lane & 16u;
-  uint32_t* bitmap = scratch + h * RFOR_HALF_WORDS;
-  uint32_t* V = bitmap + 16;
-  const uint32_t tl = C.round_base + 2u * g.cw + h;
-  const bool tv = C.t0s + tl < C.tile_end;
-  bitmap[t] = 0u;
-  const uint32_t* bV = vv.sd;
-  const uint32_t* bL = vl.sd;
-  uint32_t r = 0u, refV = 0u, refL = 0u, bvt = 0u, blt = 0u;
-  if (tv) {
-    bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
-    bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
-    r = min(bV[0], 512u);  // run / value count
-    refV = bV[1];          // references (FOR on both arrays)
-    refL = bL[1];
-    // bitwidth byte t = miniblock t (R2, R17)
-    bvt = min((bV[2 + (t >> 2)] >> (8u * (t & 3u))) & 255u, 32u);
-    blt = min((bL[2 + (t >> 2)] >> (8u * (t & 3u))) & 255u, 32u);
-  }
-  // word offset of miniblock t: every earlier miniblock is full (b_i words), R17
-  const uint32_t offv = seg16_inclusive_scan(bvt) - bvt, offl = seg16_inclusive_scan(blt) - blt;
-  __syncwarp();
-  const uint32_t rmax = max(r, __shfl_xor_sync(FULL, r, 16));
-  uint32_t carry = 0u;
-  for (uint32_t q = 0; 128u * q < rmax; ++q) {
-    const uint32_t m = 4u * q + (t >> 2);  // miniblock of this lane's 8 entries
-    const uint32_t bv = __shfl_sync(FULL, bvt, hb + m), bl = __shfl_sync(FULL, blt, hb + m);
-    const uint32_t* mV = bV + 6 + __shfl_sync(FULL, offv, hb + m);
-    const uint32_t* mL = bL + 6 + __shfl_sync(FULL, offl, hb + m);
-    const uint32_t mv = __funnelshift_lc(0xffffffffu, 0u, bv), ml = __funnelshift_lc(0xffffffffu, 0u, bl);
-    const uint32_t e0 = 128u * q + 8u * t, pos = 8u * (t & 3u);
-    uint32_t len[8], incl[8];
-    uint32_t run = 0u;
-#pragma unroll
-    for (int k = 0; k < 8; ++k) {  // 1. unpack the run lengths + local inclusive scan
-      len[k] = e0 + k < r ? refL + extract_at(mL, (pos + k) * bl, ml) : 0u;
-      run += len[k];
-      incl[k] = run;
-    }
-    // 2. 16-lane scan of the per-lane totals -> run start rows
-    const uint32_t sincl = seg16_inclusive_scan(run);
-    const uint32_t base = carry + sincl - run;
-    // 3. values to smem, run-start bits to the bitmap (predicated, branch-free)
-#pragma unroll
-    for (int k = 0; k < 8; ++k) {
-      const uint32_t S = base + incl[k] - len[k];
-      if (e0 + k < r) {
-        V[e0 + k] = refV + extract_at(mV, (pos + k) * bv, mv);
-        atomicOr(&bitmap[(S >> 5) & 15u], 1u << (S & 31u));
-      }
-    }
-    carry += __shfl_sync(FULL, sincl, hb + 15u);
-  }
-  __syncwarp();
-  // 4. expand: rows 32t .. 32t+31 of row block h
-  const uint32_t bm = bitmap[t];
-  const uint32_t pc = __popc(bm);
-  const int before = (int)(seg16_inclusive_scan(pc) - pc);  // run starts before row 32j
-#pragma unroll
-  for (int i = 0; i < 32; ++i) {
-    // row 0 of a row block always starts a run, so cur >= 0 for real rows; rows of a missing
-    // row block (no runs) read V[-1] = bitmap[15] -- in bounds, and masked by the consumer
-    const int cur = before - 1 + __popc(bm & (0xffffffffu >> (31 - i)));
-    val[i] = V[cur];
-  }
-  __syncwarp();
+  rfor_scatter_round(P, c, C, g, scratch);
+  const RforChunk k = rfor_chunk(scratch, g.lane);
+  rfor_fill(k, rfor_carry(k), val);
 }
 
 // MASK: which decoders a kernel instantiation carries (bit 1 << scheme); kernels
@@ -378,7 +426,7 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
         C.t0s = t0 + gi * TPS;
         C.stage = smem + slot * P.stage_words;
         const uint32_t nr = min(P.rounds, (t1 - C.t0s + TPR - 1) / TPR);
-        mbar_wait(&full[slot], phase);
+        if (Op::kProducerSpin) mbar_wait(&full[slot], phase); else mbar_wait_backoff(&full[slot], phase);
         for (uint32_t r = 0; r < nr; ++r, ++rc) {
           C.round_base = r * TPR;
           op.begin(P, C, g);
@@ -397,9 +445,21 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
         op.begin(P, C, g);
         for (uint32_t c = 0; c < P.ncols; ++c) {
           C.stage = smem + slot * P.stage_words;
-          mbar_wait(&full[slot], phase);
+#ifdef TP_PROFILE_WAITS
+          const long long w0 = clock64();
+#endif
+          if (Op::kProducerSpin) mbar_wait(&full[slot], phase); else mbar_wait_backoff(&full[slot], phase);
+#ifdef TP_PROFILE_WAITS
+          const long long w1 = clock64();
+#endif
           op.col(P, C, g, scratch, c, rc);
           __syncwarp();
+#ifdef TP_PROFILE_WAITS
+          if (g.lane == 0) {
+            atomicAdd(&g_prof[0], (unsigned long long)(w1 - w0));
+            atomicAdd(&g_prof[1 + min(c, 6u)], (unsigned long long)(clock64() - w1));
+          }
+#endif
           if (g.lane == 0) mbar_arrive(&empty[slot]);
           if (++slot == P.nstages) { slot = 0; phase ^= 1u; }
         }
@@ -415,6 +475,9 @@ __device__ __forceinline__ void consumers_sync() {
   asm volatile("bar.sync 1, %0;" ::"n"(CONSUMER_WARPS * 32) : "memory");
 }
 
+#ifndef TP_SPARSE_MAX
+#define TP_SPARSE_MAX 256  // alive rows (of a warp's 1024) at or below which a column goes sparse
+#endif
 #ifndef TP_QUERY_COMPACT
 #define TP_QUERY_COMPACT true
 #endif
@@ -594,23 +657,41 @@ struct SelectOp : OpBase {
 // ------------------------------------------------------------------ star-join queries
 // SSB as one tile kernel: FK columns probe dimension lookup tables
 // (Crystal's perfect hash, key - key_min), payloads build a dense group index,
-// measures are aggregated per group.  Columns come in the host's order: filters and
-// probes first (most selective first), measures last.  Grouped queries pre-aggregate
-// in a per-CTA shared-memory hash table (open addressing) and flush it once, so hot
-// groups (q4.1 has 35) do not serialise on global atomics.
+// measures are aggregated per group.  Columns come in the host's order (most selective
+// first); the last column is the aggregating measure, a first measure (MUL / SUB) is staged.
+//
+// Per column, a warp picks one of two evaluation modes (warp-uniform):
+//  * dense  -- while many of its 1024 rows are alive: decode all 32 rows per thread
+//    (tile decode) and apply the column's role to each;
+//  * sparse -- once few rows survive: visit only the alive rows and read each one's value
+//    straight out of the staged tile (random access into a FOR miniblock, Alg. 1 for one
+//    entry; for RFOR, the run whose start precedes the row) -- no work for dead rows.
+// Group index and the staged first measure live in per-warp shared memory laid out
+// [row i][lane] (conflict-free for any mix of rows).  Dense RFOR probes look each run's value
+// up once and expand the payloads (runs share their key).  Grouped queries
+// pre-aggregate in a per-CTA shared-memory hash table (open addressing) and flush it once,
+// so hot groups (q4.1 has 35) do not serialise on global atomics.
 struct StarArgs {
   int32_t role[TP_MAX_COLS], lo[TP_MAX_COLS], hi[TP_MAX_COLS];
   const int32_t* table[TP_MAX_COLS];
   int32_t key_min[TP_MAX_COLS];
   uint32_t table_len[TP_MAX_COLS], stride[TP_MAX_COLS];
+  uint32_t gmode[TP_MAX_COLS];   // probe: 0 filter only, 1 group = p * stride (first), 2 group += p * stride
+  uint32_t mstage[TP_MAX_COLS];  // measure: 1 = the first of two (staged), 0 = the aggregating one
   int agg;
   uint32_t ngroups;
-  uint32_t ht_slots, ht_shift;  // shared-memory aggregation table (grouped queries)
+  uint32_t gzero;                // grouped without payload probes: every row is group 0
+  uint32_t gs_off, ws_off;       // per-warp scratch offsets (words) of the group / staged-measure arrays
+  uint32_t ht_slots, ht_shift;   // shared-memory aggregation table (grouped queries)
+  uint32_t sparse_max;           // warp alive-row count at or below which a column is evaluated sparsely
   long long* sums;
   unsigned long long* counts;
 };
 
-constexpr uint32_t HT_MAX_SLOTS = 2048, HT_EMPTY = 0xffffffffu, HT_PROBES = 64;
+#ifndef TP_HT_MAX_SLOTS
+#define TP_HT_MAX_SLOTS 1024
+#endif
+constexpr uint32_t HT_MAX_SLOTS = TP_HT_MAX_SLOTS, HT_EMPTY = 0xffffffffu, HT_PROBES = 64;
 // slots: a power of two >= 2 x the dense group count (at most 2048); 4 words per slot:
 // key, sum lo, sum hi, count
 static inline uint32_t ht_slots(uint32_t ngroups) {
@@ -619,16 +700,20 @@ static inline uint32_t ht_slots(uint32_t ngroups) {
   return s;
 }
 
+#ifndef TP_STAR_SPIN
+#define TP_STAR_SPIN false
+#endif
 template <uint32_t MASK, bool GROUPED>
 struct StarOp : OpBase {
+  static constexpr bool kProducerSpin = TP_STAR_SPIN;
   const StarArgs* A;
   uint64_t acc, cnt;  // ungrouped (q1.x): reduce in registers
-  uint32_t alive, nmeas;
-  uint32_t gv[32];    // grouped: group index per row; ungrouped: first measure (MUL)
+  uint32_t alive;
   uint32_t* keys;
   uint32_t* hlo;   // 64-bit sums as lo/hi words: native 32-bit shared atomics with a carry
   uint32_t* hhi;   // (a 64-bit shared atomicAdd is a CAS loop on sm_100)
   uint32_t* hcnt;
+  uint32_t hmask, hshift;
 
   __device__ void cta_init(const Params& P, uint32_t* smem) {
     if (GROUPED) {
@@ -636,6 +721,8 @@ struct StarOp : OpBase {
       hlo = keys + A->ht_slots;
       hhi = keys + 2 * A->ht_slots;
       hcnt = keys + 3 * A->ht_slots;
+      hmask = A->ht_slots - 1u;
+      hshift = A->ht_shift;
       for (uint32_t i = threadIdx.x; i < A->ht_slots; i += blockDim.x) {
         keys[i] = HT_EMPTY;
         hlo[i] = 0u;
@@ -644,10 +731,8 @@ struct StarOp : OpBase {
       }
     }
   }
-  // not inlined: the caller's 32-way unrolled row loop would otherwise carry 32 copies of the
-  // probe loop and its atomics (40 % of the kernel's code, an instruction-cache thrash)
-  __device__ __noinline__ void add(uint32_t key, int64_t v, uint32_t k) {
-    uint32_t slot = (key * 0x9E3779B1u) >> A->ht_shift;  // multiplicative hash
+  __device__ __forceinline__ void ht_add(uint32_t key, int64_t v) {
+    uint32_t slot = (key * 0x9E3779B1u) >> hshift;  // multiplicative hash
 #pragma unroll 1
     for (uint32_t p = 0; p < HT_PROBES; ++p) {
       uint32_t cur = keys[slot];
@@ -660,79 +745,199 @@ struct StarOp : OpBase {
         const uint32_t old = atomicAdd(&hlo[slot], lo);
         const uint32_t carry = old + lo < old ? 1u : 0u;
         if (hi + carry) atomicAdd(&hhi[slot], hi + carry);
-        if (k) atomicAdd(&hcnt[slot], k);
+        atomicAdd(&hcnt[slot], 1u);
         return;
       }
-      slot = (slot + 1u) & (A->ht_slots - 1u);
+      slot = (slot + 1u) & hmask;
     }
     atomicAdd(reinterpret_cast<unsigned long long*>(A->sums) + key, (unsigned long long)v);  // table crowded
-    if (k) atomicAdd(A->counts + key, (unsigned long long)k);
+    atomicAdd(A->counts + key, 1ull);
   }
-  __device__ void begin(const Params& P, const StageCtx& C, const Lane& g) {
-    alive = valid_rows(P, C, g);
-    nmeas = 0;
-    if (GROUPED) {
-#pragma unroll
-      for (int i = 0; i < 32; ++i) gv[i] = 0u;
+  __device__ void begin(const Params& P, const StageCtx& C, const Lane& g) { alive = valid_rows(P, C, g); }
+
+  // the role of column c applied to row i (value x) -- shared by both modes
+  __device__ __forceinline__ void apply_range(uint32_t c, uint32_t i, uint32_t x) {
+    if ((uint32_t)((int32_t)x - A->lo[c]) > (uint32_t)(A->hi[c] - A->lo[c])) alive &= ~(1u << i);
+  }
+  __device__ __forceinline__ void apply_payload(uint32_t c, uint32_t i, int32_t p, uint32_t* G, uint32_t lane) {
+    if (p < 0) {
+      alive &= ~(1u << i);
+    } else if (GROUPED && A->gmode[c]) {
+      uint32_t* gp = G + 32u * i + lane;
+      *gp = (A->gmode[c] == 1 ? 0u : *gp) + (uint32_t)p * A->stride[c];
     }
   }
+  // payloads p[i] (-1 = miss) of the alive rows: one lean pass, warp-uniform values hoisted
+  __device__ __forceinline__ void dense_payload(uint32_t c, const uint32_t (&p)[32], uint32_t* G, uint32_t lane) {
+    uint32_t miss = 0u;
+#pragma unroll
+    for (int i = 0; i < 32; ++i) miss |= (p[i] >> 31) << i;
+    alive &= ~miss;
+    // dead rows' group entries are never read again: write all 32 (no per-row branch)
+    if (GROUPED && A->gmode[c] == 1) {
+      const uint32_t stride = A->stride[c];
+#pragma unroll
+      for (int i = 0; i < 32; ++i) G[32u * i + lane] = p[i] * stride;
+    } else if (GROUPED && A->gmode[c] == 2) {
+      const uint32_t stride = A->stride[c];
+#pragma unroll
+      for (int i = 0; i < 32; ++i) G[32u * i + lane] += p[i] * stride;
+    }
+  }
+  __device__ __forceinline__ void apply_measure(uint32_t c, uint32_t i, uint32_t x, const uint32_t* G, uint32_t* W,
+                                                uint32_t lane) {
+    if ((uint32_t)((int32_t)x - A->lo[c]) > (uint32_t)(A->hi[c] - A->lo[c])) {  // the measure's own filter
+      alive &= ~(1u << i);
+      return;
+    }
+    if (A->mstage[c]) {
+      W[32u * i + lane] = x;
+      return;
+    }
+    int64_t y = (int32_t)x;
+    if (A->agg == TP_AGG_MUL) y *= (int64_t)(int32_t)W[32u * i + lane];
+    else if (A->agg == TP_AGG_SUB) y = (int64_t)(int32_t)W[32u * i + lane] - y;
+    if (GROUPED) ht_add(A->gzero ? 0u : G[32u * i + lane], y);
+    else acc += (uint64_t)y;
+  }
+
   __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c, uint32_t) {
+    if (!__any_sync(FULL, alive != 0u)) return;  // nothing survives in this warp's rows: skip the decode
     const int role = A->role[c];
-    if (!__any_sync(FULL, alive != 0u)) {  // nothing survives in this warp's rows: skip the decode
-      if (role == TP_ROLE_MEASURE) ++nmeas;
-      return;
-    }
-    uint32_t v[32];
-    decode_col<MASK, TP_QUERY_COMPACT>(P, c, C, g, scratch, v);
-    if (role == TP_ROLE_PROBE) {
-      const int32_t* __restrict__ T = A->table[c];
-      const uint32_t kmin = (uint32_t)A->key_min[c], len = A->table_len[c], stride = A->stride[c];
-      // all 32 probes are issued before any result is used (the row mask is read from a
-      // snapshot, so no probe waits for the previous one: 32 L2 requests in flight)
-      const uint32_t m = alive;
-      int32_t pl[32];
+    const Col& col = P.col[c];
+    const bool rfor = (MASK & M_RFOR) && col.scheme == S_RFOR;
+    const bool dfor = (MASK & M_DFOR) && col.scheme == S_DFOR;  // prefix sums: no random access
+    uint32_t* G = scratch + A->gs_off;
+    uint32_t* W = scratch + A->ws_off;
+    const uint32_t lane = g.lane;
+    const uint32_t nal = __reduce_add_sync(FULL, __popc(alive));
+    const bool sparse =
+        !dfor && (nal <= A->sparse_max || (GROUPED && role == TP_ROLE_MEASURE && !A->mstage[c]));
+    RforChunk k;
+    uint32_t carry = 0u;
+    if (rfor) {
+      rfor_scatter_round(P, col, C, g, scratch);
+      k = rfor_chunk(scratch, lane);
+      if (!sparse && role == TP_ROLE_PROBE) {
+        // dense RFOR probe: one lookup per run -- the run-start values of this chunk become
+        // their payloads in place, and the expansion below spreads the payloads
+        const int32_t* __restrict__ T = A->table[c];
+        const uint32_t kmin = (uint32_t)A->key_min[c], len = A->table_len[c];
+        uint32_t mm = k.mask;
+        while (mm) {
+          uint32_t pos[4], key[4];
+          bool ok[4];
 #pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        const uint32_t k = v[i] - kmin;
-        pl[i] = ((m >> i) & 1u) && k < len ? __ldg(T + k) : -1;
+          for (int q = 0; q < 4; ++q) {
+            ok[q] = mm != 0u;
+            pos[q] = rfor_a_pos(32u * k.j + (__ffs(mm) - 1u));
+            mm &= mm - 1u;
+            key[q] = ok[q] ? k.A[pos[q]] - kmin : 0xffffffffu;
+          }
+          int32_t pl[4];
+#pragma unroll
+          for (int q = 0; q < 4; ++q) pl[q] = key[q] < len ? __ldg(T + key[q]) : -1;
+#pragma unroll
+          for (int q = 0; q < 4; ++q)
+            if (ok[q]) k.A[pos[q]] = (uint32_t)pl[q];
+        }
+        __syncwarp();
       }
-#pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        if (pl[i] < 0) alive &= ~(1u << i);
-        else if (GROUPED) gv[i] += (uint32_t)pl[i] * stride;
-      }
-      return;
+      carry = rfor_carry(k);
     }
-    const int32_t l = A->lo[c], h = A->hi[c];  // RANGE, or the measure's own filter
+    if (!sparse) {
+      // ---------------- dense: every row of the warp's round
+      uint32_t v[32];
+      if (rfor) rfor_fill(k, carry, v);
+      else decode_col<MASK & ~M_RFOR, TP_QUERY_COMPACT>(P, c, C, g, scratch, v);
+      if (role == TP_ROLE_RANGE) {
 #pragma unroll
-    for (int i = 0; i < 32; ++i)
-      if ((int32_t)v[i] < l || (int32_t)v[i] > h) alive &= ~(1u << i);
-    if (role == TP_ROLE_RANGE) return;
-    // measure
-    if (GROUPED) {
-      const bool neg = nmeas == 1;  // TP_AGG_SUB's second measure (MUL is not grouped)
+        for (int i = 0; i < 32; ++i) apply_range(c, i, v[i]);
+      } else if (role == TP_ROLE_PROBE) {
+        if (!rfor) {
+          // all 32 probes are issued before any result is used (32 L2 requests in flight)
+          const int32_t* __restrict__ T = A->table[c];
+          const uint32_t kmin = (uint32_t)A->key_min[c], len = A->table_len[c];
+          const uint32_t m = alive;
 #pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        if (alive & (1u << i)) {
-          const int64_t x = (int32_t)v[i];
-          add(gv[i], neg ? -x : x, neg ? 0u : 1u);
+          for (int i = 0; i < 32; ++i) {
+            const uint32_t kk = v[i] - kmin;
+            v[i] = ((m >> i) & 1u) && kk < len ? (uint32_t)__ldg(T + kk) : 0xffffffffu;
+          }
+        }
+        dense_payload(c, v, G, lane);
+      } else {
+        // measure: its own filter, then stage it (first of two) or aggregate it (ungrouped;
+        // grouped aggregating measures always take the sparse path)
+        const int32_t lo = A->lo[c];
+        const uint32_t span = (uint32_t)(A->hi[c] - lo);
+#pragma unroll
+        for (int i = 0; i < 32; ++i)
+          if ((uint32_t)((int32_t)v[i] - lo) > span) alive &= ~(1u << i);
+        if (A->mstage[c]) {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) W[32u * i + lane] = v[i];
+        } else if (!GROUPED) {
+          const uint32_t m = alive;
+          if (A->agg == TP_AGG_MUL) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i)
+              if (m & (1u << i)) acc += (uint64_t)((int64_t)(int32_t)v[i] * (int32_t)W[32u * i + lane]);
+          } else {
+            const bool sub = A->agg == TP_AGG_SUB;
+#pragma unroll
+            for (int i = 0; i < 32; ++i) {
+              const int64_t y = sub ? (int64_t)(int32_t)W[32u * i + lane] - (int32_t)v[i] : (int64_t)(int32_t)v[i];
+              if (m & (1u << i)) acc += (uint64_t)y;
+            }
+          }
         }
       }
-    } else if (nmeas == 0 && A->agg == TP_AGG_MUL) {
+      return;
+    }
+    // ---------------- sparse: alive rows only, values read out of the staged tile
+    MbView mv;
+    uint32_t bmask = 0u;
+    if (!rfor) {
+      const StreamView sv = stream_view(P, col.s0, C);
+      uint32_t tl;
+      bool tv;
+      mv = for_mb(P, col, C, g, sv, tl, tv);
+      bmask = __funnelshift_lc(0xffffffffu, 0u, mv.b);
+    }
+    uint32_t m = alive;
+    while (m) {
+      uint32_t ii[4], xx[4];
+      bool ok[4];
 #pragma unroll
-      for (int i = 0; i < 32; ++i) gv[i] = v[i];
-    } else {
-      const bool mul = A->agg == TP_AGG_MUL, neg = nmeas == 1 && A->agg == TP_AGG_SUB;
+      for (int q = 0; q < 4; ++q) {
+        ok[q] = m != 0u;
+        ii[q] = ok[q] ? __ffs(m) - 1u : 0u;
+        m &= m - 1u;
+        xx[q] = rfor ? rfor_row(k, carry, ii[q]) : mv.ref + extract_at(mv.w, ii[q] * mv.b, bmask);  // Alg. 1, one entry
+      }
+      if (role == TP_ROLE_RANGE) {
 #pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        if (alive & (1u << i)) {
-          int64_t x = (int32_t)v[i];
-          if (mul) x *= (int64_t)(int32_t)gv[i];
-          acc += (uint64_t)(neg ? -x : x);
+        for (int q = 0; q < 4; ++q)
+          if (ok[q]) apply_range(c, ii[q], xx[q]);
+      } else if (role == TP_ROLE_PROBE) {
+        const int32_t* __restrict__ T = A->table[c];
+        const uint32_t kmin = (uint32_t)A->key_min[c], len = A->table_len[c];
+        int32_t pl[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const uint32_t kk = xx[q] - kmin;
+          pl[q] = ok[q] && kk < len ? __ldg(T + kk) : -1;
         }
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (ok[q]) apply_payload(c, ii[q], pl[q], G, lane);
+      } else {
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (ok[q]) apply_measure(c, ii[q], xx[q], G, W, lane);
       }
     }
-    ++nmeas;
   }
   __device__ void end(const Params&, const StageCtx&, const Lane&) {
     if (!GROUPED) cnt += __popc(alive);
@@ -791,15 +996,17 @@ __global__ void __launch_bounds__(THREADS, 3)
   run_pipeline(P, op);
 }
 
+#ifndef TP_QUERY_MINB
+#define TP_QUERY_MINB 3
+#endif
 template <uint32_t MASK, bool GROUPED>
-__global__ void __launch_bounds__(THREADS, 3)
+__global__ void __launch_bounds__(THREADS, TP_QUERY_MINB)
     k_star_query(const __grid_constant__ Params P, const __grid_constant__ StarArgs A) {
   StarOp<MASK, GROUPED> op;
   op.A = &A;
   op.acc = 0;
   op.cnt = 0;
   op.alive = 0;
-  op.nmeas = 0;
   run_pipeline(P, op);
 }
 
@@ -1142,37 +1349,43 @@ tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int nc
                         uint64_t* d_counts, uint32_t ngroups, void* stream) {
   if (!dcols || !roles || !d_sums || !d_counts || ncols < 1 || ncols > TP_MAX_COLS || ngroups < 1) return TP_EINVAL;
   if (agg < TP_AGG_SUM || agg > TP_AGG_SUB) return TP_EINVAL;
-  if (agg == TP_AGG_MUL && ngroups > 1) return TP_EUNSUPPORTED;  // products are aggregated ungrouped (q1.x)
   int nmeas = 0;
   for (int c = 0; c < ncols; ++c) {
     const tp_star_col& r = roles[c];
     if (r.role < TP_ROLE_RANGE || r.role > TP_ROLE_MEASURE) return TP_EINVAL;
     if (r.role == TP_ROLE_PROBE && (!r.table || r.table_len == 0)) return TP_EINVAL;
-    if (r.role == TP_ROLE_MEASURE) {
-      // with SUB the first measure's contribution is added before the second is read
-      if (nmeas == 1 && agg == TP_AGG_SUB && (r.lo != INT_MIN || r.hi != INT_MAX)) return TP_EINVAL;
-      ++nmeas;
-    } else if (nmeas) {
-      return TP_EINVAL;  // measures come last
-    }
+    if (r.role == TP_ROLE_MEASURE) ++nmeas;
   }
-  if (nmeas != (agg == TP_AGG_SUM ? 1 : 2)) return TP_EINVAL;
+  // the last column aggregates; with MUL / SUB one earlier measure is staged
+  if (roles[ncols - 1].role != TP_ROLE_MEASURE || nmeas != (agg == TP_AGG_SUM ? 1 : 2)) return TP_EINVAL;
   if (dcols[0].n == 0) return TP_OK;
   const bool grouped = ngroups > 1;
-  Params P;
-  size_t smem = 0;
-  const uint32_t hts = grouped ? ht_slots(ngroups) : 0u;
-  tp_status st = build_params(dcols, ncols, 0, 4u * hts, P, smem);
-  if (st != TP_OK) return st;
   StarArgs A;
   memset(&A, 0, sizeof(A));
+  bool gseen = false;
   for (int c = 0; c < ncols; ++c) {
     A.role[c] = roles[c].role; A.lo[c] = roles[c].lo; A.hi[c] = roles[c].hi;
     A.table[c] = roles[c].table; A.key_min[c] = roles[c].key_min;
     A.table_len[c] = roles[c].table_len; A.stride[c] = roles[c].stride;
+    if (roles[c].role == TP_ROLE_PROBE && grouped && roles[c].stride) {
+      A.gmode[c] = gseen ? 2u : 1u;
+      gseen = true;
+    }
+    A.mstage[c] = roles[c].role == TP_ROLE_MEASURE && c != ncols - 1;
   }
+  A.gzero = grouped && !gseen;
   A.agg = agg;
   A.ngroups = ngroups;
+  A.sparse_max = TP_SPARSE_MAX;
+  if (const char* e = getenv("TILEPACK_SPARSE_MAX")) A.sparse_max = (uint32_t)atoi(e);  // tests: force a mode
+  const uint32_t hts = grouped ? ht_slots(ngroups) : 0u;
+  const uint32_t gwords = grouped ? 32u * 32u : 0u, wwords = nmeas == 2 ? 32u * 32u : 0u;
+  Params P;
+  size_t smem = 0;
+  tp_status st = build_params(dcols, ncols, gwords + wwords, 4u * hts, P, smem);
+  if (st != TP_OK) return st;
+  A.gs_off = P.staging_off;
+  A.ws_off = P.staging_off + gwords;
   A.ht_slots = hts;
   A.ht_shift = 32u - (uint32_t)__builtin_ctz(hts ? hts : 1u);
   A.sums = reinterpret_cast<long long*>(d_sums);
@@ -1197,6 +1410,14 @@ tp_status tp_plain_sum(const int32_t* d_x, uint64_t n, int64_t* d_sum, void* str
 }
 
 uint64_t tp_launch_count(void) { return g_launches.load(); }
+
+/* profiling builds (-DTP_PROFILE_WAITS): copy out and reset the cycle counters */
+tp_status tp_debug_counters(uint64_t* out16) {
+  if (cudaMemcpyFromSymbol(out16, g_prof, sizeof(unsigned long long) * 16) != cudaSuccess) return TP_ECUDA;
+  static const unsigned long long zero[16] = {0};
+  if (cudaMemcpyToSymbol(g_prof, zero, sizeof(zero)) != cudaSuccess) return TP_ECUDA;
+  return TP_OK;
+}
 
 tp_status tp_device_info(int* sms, int* ctas_per_sm) {
   if (sms) *sms = sm_count();

@@ -122,8 +122,10 @@ class SSBEngine:
             else:
                 r = self._date_range((dd["d_weeknuminyear"] == 6) & (dd["d_year"] == 1994))
                 q, dl = (26, 35), (5, 7)
-            cols = [("lo_orderdate", "range", r), ("lo_quantity", "range", q),
-                    ("lo_discount", "measure", dl), ("lo_extendedprice", "measure", None)]
+            # most selective first: the date range (RFOR, decoded whole), then the discount
+            # (the staged first measure with its filter), the quantity, the price
+            cols = [("lo_orderdate", "range", r), ("lo_discount", "measure", dl),
+                    ("lo_quantity", "range", q), ("lo_extendedprice", "measure", None)]
             return {"cols": cols, "agg": "mul", "radix": [], "decode": lambda g: ()}
         year_all = ("date", [("d_year", (1992, 1998))], "year_idx")
         if qid.startswith("2."):

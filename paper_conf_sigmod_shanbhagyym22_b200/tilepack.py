@@ -85,6 +85,7 @@ def _load():
         "tp_star_query": (i32, [colp, ctypes.POINTER(tp_star_col), i32, i32, vp, vp, u32, vp]),
         "tp_status_string": (ctypes.c_char_p, [i32]),
         "tp_launch_count": (u64, []),
+        "tp_debug_counters": (i32, [vp]),
         "tp_device_info": (i32, [vp, vp]),
     }
     for name, (res, args) in sig.items():
@@ -212,6 +213,14 @@ def decode_cascaded(dcol: "DeviceColumn", out=None, work=None, stream=None):
 
 def tp_plain_sum(d_x, n: int, d_sum, stream=None):
     _check(_lib.tp_plain_sum(_ptr(d_x), n, _ptr(d_sum), _stream(stream)), "tp_plain_sum")
+
+
+def tp_debug_counters():
+    """16 cycle counters of a -DTP_PROFILE_WAITS build (zeros otherwise); resets them."""
+    import numpy as np
+    out = np.zeros(16, np.uint64)
+    _check(_lib.tp_debug_counters(out.ctypes.data), "tp_debug_counters")
+    return out
 
 
 def tp_launch_count() -> int:
