@@ -17,6 +17,7 @@
 //     feed the consumer directly (no intermediate global pass).
 #pragma once
 #include <cstdint>
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 namespace tp {
@@ -29,7 +30,7 @@ constexpr int THREADS = 32 * (CONSUMER_WARPS + 1);
 constexpr int MAX_STREAMS = 2 * 6;  // up to 6 columns, 2 streams each (RFOR)
 constexpr unsigned FULL = 0xffffffffu;
 
-enum : uint32_t { S_FOR = 1, S_DFOR = 2, S_RFOR = 3 };
+enum : uint32_t { S_FOR = 1, S_DFOR = 2, S_RFOR = 3, S_NONE = 4 };
 
 // ------------------------------------------------------------------ PTX wrappers
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -110,6 +111,15 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
   asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
   return p;
 }
+// 2-D TMA tensor load global -> shared (UTMALDG), completes on the mbarrier
+__device__ __forceinline__ void tma_load_2d(void* dst, const void* tmap, int c0, int c1, uint64_t* bar,
+                                            uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, {%2, "
+      "%3}], [%4], %5;" ::"r"(smem_u32(dst)),
+      "l"(tmap), "r"(c0), "r"(c1), "r"(smem_u32(bar)), "l"(policy)
+      : "memory");
+}
 // 2-D TMA tensor store shared -> global (UTMASTG) and its bulk-group bookkeeping
 __device__ __forceinline__ void tma_store_2d(const void* tmap, const void* src, int c0, int c1) {
   asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(tmap),
@@ -128,7 +138,7 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 
 // ------------------------------------------------------------------ column params
 // One stream of an encoded column as the kernels see it (host fills).
-enum : uint32_t { K_FOR = 0, K_DFOR = 1, K_RFOR = 2 };  // stream kinds
+enum : uint32_t { K_FOR = 0, K_DFOR = 1, K_RFOR = 2, K_NONE = 3 };  // stream kinds
 struct Stream {
   const uint32_t* data;
   const uint32_t* starts;
@@ -142,7 +152,8 @@ struct Col {
   uint32_t nblocks;     // entries of block_starts minus one
   uint32_t s0, s1;      // indices into Params::st (s1 only for RFOR)
 };
-struct Params {
+struct alignas(64) Params {
+  CUtensorMap tmap[6];  // K_NONE columns: [rows/32][32] int32 view, 128B swizzle (TMA tensor loads)
   Stream st[MAX_STREAMS];
   Col col[6];
   uint32_t nstreams, ncols;

@@ -176,7 +176,10 @@ struct Sizes {
 
 Sizes compute_sizes(int scheme, const int32_t* x, uint64_t n) {
   Sizes s;
-  if (scheme == TP_FOR) {
+  if (scheme == TP_NONE) {  // plain values, 512-row tiles, padded to whole 32-row miniblocks
+    s.nb = (n + kTile - 1) / kTile;
+    s.w0 = (n + 31) / 32 * 32;
+  } else if (scheme == TP_FOR) {
     s.nb = (n + kBlock - 1) / kBlock;
     s.u0.resize(s.nb);
     parallel_for(s.nb, [&](uint64_t lo, uint64_t hi) {
@@ -227,7 +230,7 @@ extern "C" {
 
 tp_status tp_encode_size(int scheme, const int32_t* x, uint64_t n, uint64_t* num_blocks, uint64_t* words0,
                          uint64_t* words1) {
-  if (scheme < TP_FOR || scheme > TP_RFOR || (n && !x)) return TP_EINVAL;
+  if (scheme < TP_FOR || scheme > TP_NONE || (n && !x)) return TP_EINVAL;
   if (n >= (1ull << 32)) return TP_EUNSUPPORTED;
   Sizes s = compute_sizes(scheme, x, n);
   if (s.w0 >= (1ull << 32) || s.w1 >= (1ull << 32)) return TP_EUNSUPPORTED;
@@ -239,7 +242,7 @@ tp_status tp_encode_size(int scheme, const int32_t* x, uint64_t n, uint64_t* num
 
 tp_status tp_encode(int scheme, const int32_t* x, uint64_t n, uint32_t* starts0, uint32_t* data0, uint32_t* starts1,
                     uint32_t* data1, tp_column* out) {
-  if (scheme < TP_FOR || scheme > TP_RFOR || (n && !x) || !starts0 || !data0 || !out) return TP_EINVAL;
+  if (scheme < TP_FOR || scheme > TP_NONE || (n && !x) || !starts0 || !data0 || !out) return TP_EINVAL;
   if (scheme == TP_RFOR && (!starts1 || !data1)) return TP_EINVAL;
   if (n >= (1ull << 32)) return TP_EUNSUPPORTED;
   Sizes s = compute_sizes(scheme, x, n);
@@ -251,7 +254,19 @@ tp_status tp_encode(int scheme, const int32_t* x, uint64_t n, uint32_t* starts0,
   out->n = n;
   out->num_blocks = s.nb;
   uint32_t mtw0 = 0, mtw1 = 0;
-  if (scheme == TP_FOR) {
+  if (scheme == TP_NONE) {
+    parallel_for(s.nb, [&](uint64_t lo, uint64_t hi) {
+      for (uint64_t k = lo; k < hi; ++k) {
+        const uint64_t r0 = k * kTile, r1 = std::min<uint64_t>(n, r0 + kTile);
+        starts0[k] = (uint32_t)r0;
+        memcpy(data0 + r0, x + r0, (r1 - r0) * 4);
+      }
+    });
+    memset(data0 + n, 0, (s.w0 - n) * 4);
+    starts0[s.nb] = (uint32_t)s.w0;
+    mtw0 = kTile;
+    out->block_size = kTile; out->miniblock_count = 1; out->tile_blocks = 1;
+  } else if (scheme == TP_FOR) {
     parallel_for(s.nb, [&](uint64_t lo, uint64_t hi) {
       for (uint64_t i = lo; i < hi; ++i) {
         const uint32_t cnt = (uint32_t)std::min<uint64_t>(kBlock, n - i * kBlock);
@@ -332,6 +347,7 @@ tp_status tp_choose_scheme(const int32_t* x, uint64_t n, int* scheme, uint64_t* 
 uint64_t tp_compressed_bytes(const tp_column* c) {
   if (!c) return 0;
   const uint64_t streams = c->scheme == TP_RFOR ? 2 : 1;
+  if (c->scheme == TP_NONE) return 4 * c->n;  // the plain column (header / starts: pipeline artefacts)
   return 4 * (3 + streams * (c->num_blocks + 1) + c->words0 + c->words1);
 }
 
@@ -341,7 +357,7 @@ tp_status tp_shard(const tp_column* c, uint64_t row_lo, uint64_t row_hi, uint32_
   if (row_hi != c->n && (row_hi % kTile)) return TP_EINVAL;
   const bool rf = c->scheme == TP_RFOR;
   if (rf && !r1) return TP_EINVAL;
-  const uint64_t per = rf ? kTile : kBlock;
+  const uint64_t per = (rf || c->scheme == TP_NONE) ? kTile : kBlock;
   const uint64_t b0 = row_lo / per, b1 = (row_hi + per - 1) / per;
   *view = *c;
   view->n = row_hi - row_lo;

@@ -46,6 +46,12 @@ struct StreamView {
 __device__ __forceinline__ StreamView stream_view(const Params& P, uint32_t s, const StageCtx& C) {
   const Stream& st = P.st[s];
   StreamView v;
+  if (st.kind == K_NONE) {  // a TMA tensor box: rows of 32 words, no block_starts copy
+    v.sd = C.stage + st.data_off;
+    v.ss = v.sd;
+    v.lo = v.dshift = v.sshift = 0u;
+    return v;
+  }
   const uint32_t sidx = st.kind == K_RFOR ? C.t0s : 4u * C.t0s;
   v.ss = C.stage + st.starts_off;
   v.sd = C.stage + st.data_off;
@@ -293,9 +299,32 @@ __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const
   rfor_fill(k, rfor_carry(k), val);
 }
 
+// ---------------------------------------------------------------- None (uncompressed)
+// The plain column staged as a 128B-swizzled TMA box of 32-word rows: row r = 16 * tile + mb
+// holds the thread's 32 values, 16-byte chunk q at chunk q ^ (r & 7).
+__device__ __forceinline__ const uint32_t* none_row(const Params& P, const Col& c, const StageCtx& C,
+                                                    const Lane& g, uint32_t& sw) {
+  const uint32_t r = 16u * (C.round_base + g.tile_local) + g.mb;
+  sw = r & 7u;
+  return C.stage + P.st[c.s0].data_off + 32u * r;
+}
+__device__ __forceinline__ void decode_none(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
+                                            uint32_t (&val)[32]) {
+  uint32_t sw;
+  const uint32_t* w = none_row(P, c, C, g, sw);
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const uint4 a = *reinterpret_cast<const uint4*>(w + ((q ^ sw) << 2));
+    val[4 * q] = a.x; val[4 * q + 1] = a.y; val[4 * q + 2] = a.z; val[4 * q + 3] = a.w;
+  }
+}
+__device__ __forceinline__ uint32_t none_at(const uint32_t* w, uint32_t sw, uint32_t i) {
+  return w[((((i >> 2) ^ sw) << 2)) | (i & 3u)];
+}
+
 // MASK: which decoders a kernel instantiation carries (bit 1 << scheme); kernels
 // are instantiated per scheme mix so that FOR-only kernels keep FOR's register budget.
-constexpr uint32_t M_FOR = 1u << S_FOR, M_DFOR = 1u << S_DFOR, M_RFOR = 1u << S_RFOR;
+constexpr uint32_t M_FOR = 1u << S_FOR, M_DFOR = 1u << S_DFOR, M_RFOR = 1u << S_RFOR, M_NONE = 1u << S_NONE;
 constexpr uint32_t M_RAW = 1u << 8;  // FOR / DFOR blocks, packed offsets only (cascading baseline)
 template <uint32_t MASK, bool COMPACT = false>
 __device__ __forceinline__ void decode_col(const Params& P, uint32_t ci, const StageCtx& C, const Lane& g,
@@ -305,7 +334,8 @@ __device__ __forceinline__ void decode_col(const Params& P, uint32_t ci, const S
     decode_for<false, true>(P, c, C, g, val);
     return;
   }
-  if ((MASK & M_FOR) && c.scheme == S_FOR) decode_for<COMPACT>(P, c, C, g, val);
+  if ((MASK & M_NONE) && c.scheme == S_NONE) decode_none(P, c, C, g, val);
+  else if ((MASK & M_FOR) && c.scheme == S_FOR) decode_for<COMPACT>(P, c, C, g, val);
   else if ((MASK & M_DFOR) && c.scheme == S_DFOR) decode_dfor<COMPACT>(P, c, C, g, val);
   else if (MASK & M_RFOR) decode_rfor(P, c, C, g, scratch, val);
 }
@@ -383,7 +413,12 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
           uint32_t bytes = 0u, dbytes = 0u, sbytes = 0u;
           const char *dsrc = nullptr, *ssrc = nullptr;
           uint32_t *dst_d = nullptr, *dst_s = nullptr;
-          if (my_s != 0xffu) {
+          const bool none = my_s != 0xffu && P.st[my_s].kind == K_NONE;
+          if (none) {  // plain column: one TMA tensor box of TPS tiles (OOB rows zero-filled)
+            dbytes = TPS * TILE_ROWS * 4u;
+            bytes = dbytes;
+            dst_d = smem + slot * P.stage_words + P.st[my_s].data_off;
+          } else if (my_s != 0xffu) {
             const Stream& st = P.st[my_s];
             const uint32_t lo = mylo - (st.kind == K_DFOR ? 1u : 0u);
             const uintptr_t a0 = reinterpret_cast<uintptr_t>(st.data + lo) & ~uintptr_t(15);
@@ -404,7 +439,9 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
           const uint32_t total = __reduce_add_sync(FULL, bytes);
           if (lane == 0) mbar_arrive_expect_tx(&full[slot], total);
           __syncwarp();
-          if (my_s != 0xffu) {
+          if (none) {
+            tma_load_2d(dst_d, &P.tmap[c], 0, (int)(tile_base * (TILE_ROWS / 32)), &full[slot], pol);
+          } else if (my_s != 0xffu) {
             bulk_g2s(dst_d, dsrc, dbytes, &full[slot], pol);
             bulk_g2s(dst_s, ssrc, sbytes, &full[slot], pol);
           }
@@ -897,8 +934,12 @@ struct StarOp : OpBase {
     }
     // ---------------- sparse: alive rows only, values read out of the staged tile
     MbView mv;
-    uint32_t bmask = 0u;
-    if (!rfor) {
+    uint32_t bmask = 0u, nsw = 0u;
+    const bool none = (MASK & M_NONE) && col.scheme == S_NONE;
+    const uint32_t* nw = nullptr;
+    if (none) {
+      nw = none_row(P, col, C, g, nsw);
+    } else if (!rfor) {
       const StreamView sv = stream_view(P, col.s0, C);
       uint32_t tl;
       bool tv;
@@ -914,7 +955,9 @@ struct StarOp : OpBase {
         ok[q] = m != 0u;
         ii[q] = ok[q] ? __ffs(m) - 1u : 0u;
         m &= m - 1u;
-        xx[q] = rfor ? rfor_row(k, carry, ii[q]) : mv.ref + extract_at(mv.w, ii[q] * mv.b, bmask);  // Alg. 1, one entry
+        xx[q] = none ? none_at(nw, nsw, ii[q])
+                : rfor ? rfor_row(k, carry, ii[q])
+                       : mv.ref + extract_at(mv.w, ii[q] * mv.b, bmask);  // Alg. 1, one entry
       }
       if (role == TP_ROLE_RANGE) {
 #pragma unroll
@@ -1071,7 +1114,20 @@ static int sm_count() {
 #ifndef TP_QUERY_RING_KB
 #define TP_QUERY_RING_KB 24
 #endif
+static PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  }
+  return fn;
+}
+
 static uint32_t worst_tile_words(uint32_t scheme) {
+  if (scheme == TP_NONE) return TILE_ROWS;
   return scheme == TP_FOR ? 4u * (2u + 128u) : scheme == TP_DFOR ? 1u + 4u * (2u + 128u) : 6u + 512u;
 }
 static uint32_t align4(uint32_t w) { return (w + 3u) & ~3u; }
@@ -1086,7 +1142,7 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
   if (!cols || ncols < 1 || ncols > TP_MAX_COLS) return TP_EINVAL;
   const uint64_t n = cols[0].n;
   if (n >= (1ull << 32)) return TP_EUNSUPPORTED;
-  bool any_rfor = false;
+  bool any_rfor = false, any_none = false;
   uint32_t mtws[MAX_STREAMS];
   uint32_t max_round_words = 0;  // data words of one round (TPR tiles) of the widest column
   for (int c = 0; c < ncols; ++c) {
@@ -1094,7 +1150,10 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
     if (k.n != n) return TP_EINVAL;
     if (k.words0 >= (1ull << 32) || k.words1 >= (1ull << 32)) return TP_EUNSUPPORTED;
     const bool rf = k.scheme == TP_RFOR;
-    if (k.scheme == TP_FOR || k.scheme == TP_DFOR) {
+    if (k.scheme == TP_NONE) {
+      if (k.block_size != 512 || k.num_blocks != (n + 511) / 512 || k.words0 < n) return TP_EFORMAT;
+      if (reinterpret_cast<uintptr_t>(k.data0) & 15u) return TP_EINVAL;
+    } else if (k.scheme == TP_FOR || k.scheme == TP_DFOR) {
       if (k.block_size != 128 || k.miniblock_count != 4 || k.num_blocks != (n + 127) / 128) return TP_EFORMAT;
     } else if (rf) {
       if (k.block_size != 512 || k.miniblock_count != 16 || k.num_blocks != (n + 511) / 512) return TP_EFORMAT;
@@ -1105,17 +1164,35 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
     if (n > 0 && (!k.starts0 || !k.data0)) return TP_EINVAL;
     any_rfor |= rf;
     Col& cc = P.col[c];
-    cc.scheme = k.scheme == TP_FOR ? S_FOR : k.scheme == TP_DFOR ? S_DFOR : S_RFOR;
+    cc.scheme = k.scheme == TP_FOR ? S_FOR : k.scheme == TP_DFOR ? S_DFOR : k.scheme == TP_RFOR ? S_RFOR : S_NONE;
     cc.nblocks = (uint32_t)k.num_blocks;
     uint32_t rw = 0;
     for (int s = 0; s < (rf ? 2 : 1); ++s) {
       Stream& st = P.st[P.nstreams];
       st.data = s == 0 ? k.data0 : k.data1;
       st.starts = s == 0 ? k.starts0 : k.starts1;
-      st.kind = rf ? K_RFOR : (k.scheme == TP_DFOR ? K_DFOR : K_FOR);
+      st.kind = rf ? K_RFOR : k.scheme == TP_DFOR ? K_DFOR : k.scheme == TP_NONE ? K_NONE : K_FOR;
       st.nblocks = (uint32_t)k.num_blocks;
       uint32_t mtw = s == 0 ? k.max_tile_words0 : k.max_tile_words1;
       if (mtw == 0 || mtw > worst_tile_words(k.scheme)) mtw = worst_tile_words(k.scheme);
+      if (k.scheme == TP_NONE) {
+        mtw = TILE_ROWS;
+        any_none = true;
+        // [words0 / 32][32] int32 tensor, boxes of 16 rows per tile, 128-byte swizzle (the
+        // consumers' 16-byte reads of a 32-row miniblock are then bank-conflict free)
+        if (n > 0) {
+          auto enc = tensor_map_encoder();
+          if (!enc) return TP_ECUDA;
+          cuuint64_t dims[2] = {32, (cuuint64_t)(k.words0 / 32)};
+          cuuint64_t strides[1] = {128};
+          cuuint32_t box[2] = {32, (cuuint32_t)(TPR * (TILE_ROWS / 32))};
+          cuuint32_t estr[2] = {1, 1};
+          if (enc(&P.tmap[c], CU_TENSOR_MAP_DATA_TYPE_INT32, 2, const_cast<uint32_t*>(k.data0), dims, strides, box,
+                  estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+            return TP_ECUDA;
+        }
+      }
       mtws[P.nstreams] = mtw;
       rw += TPR * mtw;
       if (s == 0) cc.s0 = P.nstreams; else cc.s1 = P.nstreams;
@@ -1136,6 +1213,13 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
     const uint32_t q0 = P.col[c].s0, q1 = P.col[c].scheme == S_RFOR ? P.col[c].s1 : q0;
     for (uint32_t q = q0; q <= q1; ++q) {
       Stream& st = P.st[q];
+      if (st.kind == K_NONE) {  // a 1024-byte aligned swizzled box, no block_starts region
+        off = (off + 255u) & ~255u;
+        st.data_off = off;
+        off += TPS * TILE_ROWS;
+        st.starts_off = off;
+        continue;
+      }
       st.data_off = off;
       off += align4(std::max<uint32_t>(TPS * mtws[q] + 12u, 48u));  // + alignment slop + unpack over-read
       st.starts_off = off;
@@ -1146,7 +1230,7 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
   P.ncols = (uint32_t)ncols;
   P.n = (uint32_t)n;
   P.ntiles = (uint32_t)((n + TILE_ROWS - 1) / TILE_ROWS);
-  P.stage_words = align4(item);
+  P.stage_words = any_none ? (item + 255u) & ~255u : align4(item);  // NONE boxes: 1024-byte aligned
   P.staging_off = any_rfor ? RFOR_SCRATCH_WORDS : 0u;
   P.scratch_words_per_warp = align4(P.staging_off + extra_scratch);
   // ring depth: 2..8 items within ~40 KB, so that several CTAs (16+ consumer warps) share
@@ -1194,17 +1278,6 @@ static tp_status launched() {
   return cudaGetLastError() == cudaSuccess ? TP_OK : TP_ECUDA;
 }
 
-static PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
-  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
-  if (!fn) {
-    void* p = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
-        q == cudaDriverEntryPointSuccess)
-      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
-  }
-  return fn;
-}
 
 #define TP_DISPATCH_MASK(MASKV, CALL)                               \
   switch (MASKV) {                                                  \
@@ -1214,7 +1287,8 @@ static PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
     case M_FOR | M_DFOR: { constexpr uint32_t MK = M_FOR | M_DFOR; CALL; } break; \
     case M_FOR | M_RFOR: { constexpr uint32_t MK = M_FOR | M_RFOR; CALL; } break; \
     case M_DFOR | M_RFOR: { constexpr uint32_t MK = M_DFOR | M_RFOR; CALL; } break; \
-    default: { constexpr uint32_t MK = M_FOR | M_DFOR | M_RFOR; CALL; } break; \
+    case M_NONE: { constexpr uint32_t MK = M_NONE; CALL; } break;   \
+    default: { constexpr uint32_t MK = M_FOR | M_DFOR | M_RFOR | M_NONE; CALL; } break; \
   }
 
 }  // namespace tp
@@ -1235,6 +1309,7 @@ tp_status tp_decode_sum(const tp_column* dcol, int64_t* d_sum, void* stream) {
   switch (scheme_mask(P)) {
     case M_FOR: launch(k_decode_sum<M_FOR>, smem, cap, stream, P, out); break;
     case M_DFOR: launch(k_decode_sum<M_DFOR>, smem, cap, stream, P, out); break;
+    case M_NONE: launch(k_decode_sum<M_NONE>, smem, cap, stream, P, out); break;
     default: launch(k_decode_sum<M_RFOR>, smem, cap, stream, P, out); break;
   }
   return launched();
@@ -1277,6 +1352,7 @@ tp_status decode_global_impl(const tp_column* dcol, int32_t* d_out, bool raw, vo
   switch (scheme_mask(P)) {
     case M_FOR: launch(k_decode_global<M_FOR>, smem, cap, stream, P, tmap, d_out); break;
     case M_DFOR: launch(k_decode_global<M_DFOR>, smem, cap, stream, P, tmap, d_out); break;
+    case M_NONE: launch(k_decode_global<M_NONE>, smem, cap, stream, P, tmap, d_out); break;
     default: launch(k_decode_global<M_RFOR>, smem, cap, stream, P, tmap, d_out); break;
   }
   return launched();

@@ -27,6 +27,8 @@ def main():
     ap.add_argument("--check", action="store_true", help="compare every result with the oracle (rank 0)")
     ap.add_argument("--out", default=None)
     ap.add_argument("--queries", default="all")
+    ap.add_argument("--scheme", default="auto", help="auto (GPU-*, P:1206-1217) | none (uncompressed baseline, "
+                    "Fig. 11) | for | dfor | rfor for every lineorder column")
     args = ap.parse_args()
     import torch
     import torch.distributed as dist
@@ -45,7 +47,8 @@ def main():
     from paper_conf_sigmod_shanbhagyym22_b200.dist import tile_range
     r0, r1 = tile_range(n, rank, world)
     gen_s = time.time() - t0
-    eng = SSBEngine(db, dev, rows=(r0, r1))
+    from paper_conf_sigmod_shanbhagyym22_b200.ssb import QUERY_COLUMNS
+    eng = SSBEngine(db, dev, rows=(r0, r1), schemes={c: args.scheme for c in QUERY_COLUMNS})
     setup_s = time.time() - t0
     peak = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"])
     stream = torch.cuda.current_stream(dev)
@@ -109,7 +112,7 @@ def main():
             print(qid, json.dumps({k: (round(v, 4) if isinstance(v, float) else v) for k, v in r.items()}), flush=True)
         res[qid] = r
     if rank == 0:
-        summary = {"sf": args.sf, "rows": n, "n_gpus": world, "gen_s": gen_s, "setup_s": setup_s,
+        summary = {"sf": args.sf, "rows": n, "n_gpus": world, "scheme": args.scheme, "gen_s": gen_s, "setup_s": setup_s,
                    "cpu_baseline": None if oracle is None else {
                        "kind": "oracle", "cores": 1, "what": "oracle/ssb.py: numpy SQL over the uncompressed "
                        "columns, per query (oracle_s), plus a shared date join of %.2f s" % oracle_join_s},

@@ -159,3 +159,16 @@ def test_cascaded_baseline_parity(scheme):
          "rfor": datagen.runs(3_000_001, 6, seed=4)}[scheme]
     d = tp.encode(x, scheme).to_device()
     assert np.array_equal(tp.decode_cascaded(d).cpu().numpy(), x)
+
+
+@pytest.mark.parametrize("n", [1, 31, 512, 512 * 8 + 5, 512 * 37 + 77, 3_000_001])
+def test_none_plain_column(n):
+    """TP_NONE (the uncompressed baseline): decode == the column itself, through the
+    TMA tensor-box path (ragged tails zero-filled by the box, masked by the consumer)."""
+    x = np.random.default_rng(n).integers(-(2**31), 2**31, n, dtype=np.int64).astype(np.int32)
+    d = tp.encode(x, "none").to_device()
+    assert np.array_equal(tp.decode(d).cpu().numpy(), x)
+    assert int(tp.decode_sum(d).item()) == oracle.column_sum(x)
+    got = int(tp.select_project_sum([d, d], [-(2**30), 0], [2**30, 2**31 - 1], "col", 1, 0).item())
+    want = oracle.select_project_sum([x, x], [-(2**30), 0], [2**30, 2**31 - 1], "col", 1, 0)
+    assert got == want

@@ -97,3 +97,15 @@ def test_errors():
     r0 = np.zeros(64, np.uint32)
     with pytest.raises(tp.TilepackError):
         tp.tp_shard(h.col, 100, 600, r0)   # not tile aligned
+
+
+def test_none_layout():
+    """TP_NONE: block_starts = 512 k, data = the values zero-padded to 32 words, bytes = 4 n."""
+    for n in (0, 1, 511, 512, 513, 5000):
+        x = np.arange(n, dtype=np.int32) * 3 - 7
+        h = tp.encode(x, "none")
+        nb = (n + 511) // 512
+        assert int(h.col.num_blocks) == nb and int(h.col.words0) == (n + 31) // 32 * 32
+        assert list(h.starts0[:nb]) == [512 * k for k in range(nb)] and h.starts0[nb] == h.col.words0
+        assert np.array_equal(h.data0[:n].view(np.int32), x) and not h.data0[n:].any()
+        assert h.nbytes() == 4 * n

@@ -49,6 +49,11 @@ def _cases(d):
         # ungrouped SUB, measures on RFOR / DFOR columns
         (["qty", "keys", "srt"], ["for", "rfor", "dfor"],
          [dict(role="range", lo=10, hi=40), meas(), meas()], "sub", 1),
+        # the uncompressed baseline (None) mixed with compressed columns
+        (["keys", "fk", "qty", "price"], ["none", "rfor", "none", "for"],
+         [probe1, probe2, dict(role="range", lo=5, hi=30), meas()], "sum", 7 * 25),
+        (["price", "qty", "cost"], ["none", "none", "none"],
+         [meas(-(1 << 19), 1 << 23), dict(role="range", lo=1, hi=24), meas()], "mul", 1),
         # grouped MUL, filter-only probe, no payload probe -> single group 0 of 3
         (["fk", "qty", "cost"], ["for", "for", "for"],
          [dict(role="probe", table=d["t2"], key_min=0, stride=0), meas(), meas(0, 60000)], "mul", 3),
