@@ -45,13 +45,7 @@ struct StreamView {
 // the per-round critical path than sharing it through shared memory and a warp sync.
 __device__ __forceinline__ StreamView stream_view(const Params& P, uint32_t s, const StageCtx& C) {
   const Stream& st = P.st[s];
-  StreamView v;
-  if (st.kind == K_NONE) {  // a TMA tensor box: rows of 32 words, no block_starts copy
-    v.sd = C.stage + st.data_off;
-    v.ss = v.sd;
-    v.lo = v.dshift = v.sshift = 0u;
-    return v;
-  }
+  StreamView v;  // FOR / DFOR / RFOR streams only (a None column is read through none_row)
   const uint32_t sidx = st.kind == K_RFOR ? C.t0s : 4u * C.t0s;
   v.ss = C.stage + st.starts_off;
   v.sd = C.stage + st.data_off;
@@ -413,7 +407,8 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
           uint32_t bytes = 0u, dbytes = 0u, sbytes = 0u;
           const char *dsrc = nullptr, *ssrc = nullptr;
           uint32_t *dst_d = nullptr, *dst_s = nullptr;
-          const bool none = my_s != 0xffu && P.st[my_s].kind == K_NONE;
+          // compiled only into kernels that carry the None reader (keeps FOR kernels lean)
+          const bool none = (Op::kMask & M_NONE) && my_s != 0xffu && P.st[my_s].kind == K_NONE;
           if (none) {  // plain column: one TMA tensor box of TPS tiles (OOB rows zero-filled)
             dbytes = TPS * TILE_ROWS * 4u;
             bytes = dbytes;
@@ -536,6 +531,7 @@ __device__ __forceinline__ uint32_t valid_rows(const Params& P, const StageCtx& 
 
 struct OpBase {
   static constexpr bool kProducerSpin = false;
+  static constexpr uint32_t kMask = ~0u;  // scheme mix the kernel carries (M_*)
   __device__ void cta_init(const Params&, uint32_t*) {}
   __device__ void begin(const Params&, const StageCtx&, const Lane&) {}
   __device__ void end(const Params&, const StageCtx&, const Lane&) {}
@@ -544,6 +540,7 @@ struct OpBase {
 // decode -> sum (decode-only microbenchmark)
 template <uint32_t MASK>
 struct SumOp : OpBase {
+  static constexpr uint32_t kMask = MASK;
   static constexpr bool kProducerSpin = MASK == M_FOR;
   unsigned long long* out;
   uint64_t acc;
@@ -596,6 +593,7 @@ struct SumOp : OpBase {
 // one TMA tensor store; the partial last miniblock (n % 32 rows) is stored directly.
 template <uint32_t MASK>
 struct GlobalOp : OpBase {
+  static constexpr uint32_t kMask = MASK;
   static constexpr bool kProducerSpin = true;  // HBM-bound (decoded rows are written back)
   const CUtensorMap* tmap;
   int32_t* out;
@@ -648,6 +646,7 @@ struct SelectArgs {
 
 template <uint32_t MASK>
 struct SelectOp : OpBase {
+  static constexpr uint32_t kMask = MASK;
   const SelectArgs* A;
   unsigned long long* out;
   uint64_t acc;
@@ -742,6 +741,7 @@ static inline uint32_t ht_slots(uint32_t ngroups) {
 #endif
 template <uint32_t MASK, bool GROUPED>
 struct StarOp : OpBase {
+  static constexpr uint32_t kMask = MASK;
   static constexpr bool kProducerSpin = TP_STAR_SPIN;
   const StarArgs* A;
   uint64_t acc, cnt;  // ungrouped (q1.x): reduce in registers
