@@ -224,6 +224,51 @@ tp_status tp_plain_sum(const int32_t* d_x, uint64_t n, int64_t* d_sum, void* str
 uint64_t tp_cascaded_workspace_words(const tp_column* col);
 tp_status tp_decode_cascaded(const tp_column* dcol, int32_t* d_out, uint32_t* d_work, void* stream);
 
+/* ------------------------------------------------------ GPU encoder (tile-parallel)
+ * The paper compresses once on the host; every 512-row tile is encoded
+ * independently, so the encoder also runs on the GPU
+ * in one pass over a DEVICE column: warps plan and pack tiles, a decoupled look-back over
+ * 4096-row chunks gives each tile its word offset.  The bytes are
+ * identical to tp_encode's.  d_x must be 16-byte aligned.
+ *
+ * d_work: DEVICE scratch of tp_gpu_encode_workspace_bytes(n) bytes (8-byte aligned), owned
+ * by the caller; the calls zero it themselves (stream-ordered). */
+uint64_t tp_gpu_encode_workspace_bytes(uint64_t n);
+
+/* Capacity that always suffices for scheme on n rows (host arithmetic, no device work):
+ * *num_blocks as tp_encode_size; *words0 / *words1 = worst-case data words (every miniblock
+ * 32 bits wide: FOR 130 words per 128 rows, DFOR + 1 per tile, RFOR 518 per 512 rows and
+ * stream, None n rounded up to 32).  Allocate starts with num_blocks+1+TP_GUARD_WORDS words and
+ * data with words+TP_GUARD_WORDS words. */
+tp_status tp_gpu_encode_bound(int scheme, uint64_t n, uint64_t* num_blocks, uint64_t* words0, uint64_t* words1);
+
+/* Exact data words of all three formats for DEVICE d_x[0..n), one pass (GPU-* analysis,
+ * P:1206-1217): words4 (host) = {FOR, DFOR, RFOR values, RFOR run lengths}.  Blocks until
+ * the counts are on the host. */
+tp_status tp_gpu_encode_sizes(const int32_t* d_x, uint64_t n, void* d_work, uint64_t* words4, void* stream);
+
+/* GPU-* on a DEVICE column (same rule as tp_choose_scheme: smallest footprint, ties
+ * FOR < DFOR < RFOR, R20).  Blocks. */
+tp_status tp_gpu_choose_scheme(const int32_t* d_x, uint64_t n, void* d_work, int* scheme, uint64_t* bytes,
+                               void* stream);
+
+/* Encode DEVICE d_x[0..n) into DEVICE arrays: starts0/data0 (+ starts1/data1 for RFOR) as
+ * for tp_encode; cap0 / cap1 = usable data words (guards excluded; tp_gpu_encode_bound or
+ * tp_gpu_encode_sizes give a sufficient value).  Writes every used word, the last
+ * block_starts entry and the zero guard words.  tp_gpu_encode_launch is asynchronous on
+ * `stream`; tp_gpu_encode_result waits for it and fills *out with the device pointers, word
+ * counts and max_tile_words (TP_ESIZE if a capacity was too small -- the arrays are then
+ * incomplete).  tp_gpu_encode = launch + result. */
+tp_status tp_gpu_encode_launch(int scheme, const int32_t* d_x, uint64_t n, uint32_t* d_starts0, uint32_t* d_data0,
+                               uint64_t cap0, uint32_t* d_starts1, uint32_t* d_data1, uint64_t cap1, void* d_work,
+                               void* stream);
+tp_status tp_gpu_encode_result(int scheme, uint64_t n, const uint32_t* d_starts0, const uint32_t* d_data0,
+                               const uint32_t* d_starts1, const uint32_t* d_data1, const void* d_work,
+                               tp_column* out, void* stream);
+tp_status tp_gpu_encode(int scheme, const int32_t* d_x, uint64_t n, uint32_t* d_starts0, uint32_t* d_data0,
+                        uint64_t cap0, uint32_t* d_starts1, uint32_t* d_data1, uint64_t cap1, void* d_work,
+                        tp_column* out, void* stream);
+
 /* --------------------------------------------------------------- utility */
 
 const char* tp_status_string(tp_status s);

@@ -83,6 +83,13 @@ def _load():
         "tp_decode_cascaded": (i32, [colp, vp, vp, vp]),
         "tp_lookup_build": (i32, [vp, u64, ctypes.c_int32, u32, ctypes.POINTER(tp_dim_pred), i32, vp, vp, vp]),
         "tp_star_query": (i32, [colp, ctypes.POINTER(tp_star_col), i32, i32, vp, vp, u32, vp]),
+        "tp_gpu_encode_workspace_bytes": (u64, [u64]),
+        "tp_gpu_encode_bound": (i32, [i32, u64, vp, vp, vp]),
+        "tp_gpu_encode_sizes": (i32, [vp, u64, vp, vp, vp]),
+        "tp_gpu_choose_scheme": (i32, [vp, u64, vp, vp, vp, vp]),
+        "tp_gpu_encode_launch": (i32, [i32, vp, u64, vp, vp, u64, vp, vp, u64, vp, vp]),
+        "tp_gpu_encode_result": (i32, [i32, u64, vp, vp, vp, vp, vp, colp, vp]),
+        "tp_gpu_encode": (i32, [i32, vp, u64, vp, vp, u64, vp, vp, u64, vp, colp, vp]),
         "tp_status_string": (ctypes.c_char_p, [i32]),
         "tp_launch_count": (u64, []),
         "tp_debug_counters": (i32, [vp]),
@@ -211,6 +218,52 @@ def decode_cascaded(dcol: "DeviceColumn", out=None, work=None, stream=None):
     return out
 
 
+# ---- GPU encoder (tile-parallel, one pass; include/tilepack.h "GPU encoder")
+def tp_gpu_encode_workspace_bytes(n: int) -> int:
+    return int(_lib.tp_gpu_encode_workspace_bytes(n))
+
+
+def tp_gpu_encode_bound(scheme: int, n: int):
+    nb, w0, w1 = ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_uint64()
+    _check(_lib.tp_gpu_encode_bound(scheme, n, ctypes.byref(nb), ctypes.byref(w0), ctypes.byref(w1)),
+           "tp_gpu_encode_bound")
+    return nb.value, w0.value, w1.value
+
+
+def tp_gpu_encode_sizes(d_x, n: int, d_work, stream=None):
+    w = (ctypes.c_uint64 * 4)()
+    _check(_lib.tp_gpu_encode_sizes(_ptr(d_x), n, _ptr(d_work), w, _stream(stream)), "tp_gpu_encode_sizes")
+    return [int(v) for v in w]
+
+
+def tp_gpu_choose_scheme(d_x, n: int, d_work, stream=None):
+    s, b = ctypes.c_int(), ctypes.c_uint64()
+    _check(_lib.tp_gpu_choose_scheme(_ptr(d_x), n, _ptr(d_work), ctypes.byref(s), ctypes.byref(b), _stream(stream)),
+           "tp_gpu_choose_scheme")
+    return s.value, b.value
+
+
+def tp_gpu_encode_launch(scheme: int, d_x, n: int, starts0, data0, cap0: int, starts1, data1, cap1: int, d_work,
+                         stream=None):
+    _check(_lib.tp_gpu_encode_launch(scheme, _ptr(d_x), n, _ptr(starts0), _ptr(data0), cap0, _ptr(starts1),
+                                     _ptr(data1), cap1, _ptr(d_work), _stream(stream)), "tp_gpu_encode_launch")
+
+
+def tp_gpu_encode_result(scheme: int, n: int, starts0, data0, starts1, data1, d_work, stream=None) -> tp_column:
+    col = tp_column()
+    _check(_lib.tp_gpu_encode_result(scheme, n, _ptr(starts0), _ptr(data0), _ptr(starts1), _ptr(data1),
+                                     _ptr(d_work), ctypes.byref(col), _stream(stream)), "tp_gpu_encode_result")
+    return col
+
+
+def tp_gpu_encode(scheme: int, d_x, n: int, starts0, data0, cap0: int, starts1, data1, cap1: int, d_work,
+                  stream=None) -> tp_column:
+    col = tp_column()
+    _check(_lib.tp_gpu_encode(scheme, _ptr(d_x), n, _ptr(starts0), _ptr(data0), cap0, _ptr(starts1), _ptr(data1),
+                              cap1, _ptr(d_work), ctypes.byref(col), _stream(stream)), "tp_gpu_encode")
+    return col
+
+
 def tp_plain_sum(d_x, n: int, d_sum, stream=None):
     _check(_lib.tp_plain_sum(_ptr(d_x), n, _ptr(d_sum), _stream(stream)), "tp_plain_sum")
 
@@ -305,6 +358,58 @@ class DeviceColumn:
 
     def nbytes(self) -> int:
         return tp_compressed_bytes(self.col)
+
+
+class GpuColumn:
+    """A column encoded ON THE DEVICE by the tile-parallel encoder (tp_gpu_encode): torch int32
+    storage (capacity = the bound, or exact sizes with exact=True) + its tp_column of device
+    pointers.  Same interface as DeviceColumn."""
+
+    def __init__(self, x, scheme: str = "for", exact: bool = False, work=None, stream=None):
+        import torch
+        assert x.is_cuda and x.dtype == torch.int32 and x.is_contiguous()
+        n = x.numel()
+        dev = x.device
+        if work is None:
+            work = torch.empty((tp_gpu_encode_workspace_bytes(n) + 7) // 8, dtype=torch.int64, device=dev)
+        if scheme == "auto":
+            s, _ = tp_gpu_choose_scheme(x, n, work, stream)
+            scheme = SCHEME_NAMES[s]
+        sc = SCHEMES[scheme]
+        nb, w0, w1 = tp_gpu_encode_bound(sc, n)
+        if exact and sc != TP_NONE:
+            w = tp_gpu_encode_sizes(x, n, work, stream)
+            w0, w1 = {TP_FOR: (w[0], 0), TP_DFOR: (w[1], 0), TP_RFOR: (w[2], w[3])}[sc]
+        self.scheme = scheme
+        self.starts0 = torch.empty(nb + 1 + GUARD_WORDS, dtype=torch.int32, device=dev)
+        self.data0 = torch.empty(w0 + GUARD_WORDS, dtype=torch.int32, device=dev)
+        rf = sc == TP_RFOR
+        self.starts1 = torch.empty(nb + 1 + GUARD_WORDS, dtype=torch.int32, device=dev) if rf else None
+        self.data1 = torch.empty(w1 + GUARD_WORDS, dtype=torch.int32, device=dev) if rf else None
+        self.col = tp_gpu_encode(sc, x, n, self.starts0, self.data0, w0, self.starts1, self.data1, w1, work, stream)
+
+    @property
+    def n(self) -> int:
+        return int(self.col.n)
+
+    def nbytes(self) -> int:
+        return tp_compressed_bytes(self.col)
+
+    def arrays(self) -> dict:
+        """Used words only, copied to the host (the oracle's layout for byte comparison)."""
+        nb = int(self.col.num_blocks)
+        hdr = np.array([self.col.block_size, self.col.miniblock_count, self.col.n], np.uint32)
+        d = {"header": hdr, "starts0": self.starts0[:nb + 1].cpu().numpy().view(np.uint32),
+             "data0": self.data0[:self.col.words0].cpu().numpy().view(np.uint32)}
+        if self.starts1 is not None:
+            d["starts1"] = self.starts1[:nb + 1].cpu().numpy().view(np.uint32)
+            d["data1"] = self.data1[:self.col.words1].cpu().numpy().view(np.uint32)
+        return d
+
+
+def gpu_encode(x, scheme: str = "for", exact: bool = False, stream=None) -> GpuColumn:
+    """Encode a DEVICE int32 tensor on the GPU (scheme 'for' | 'dfor' | 'rfor' | 'none' | 'auto')."""
+    return GpuColumn(x, scheme, exact=exact, stream=stream)
 
 
 def encode(x: np.ndarray, scheme: str = "for") -> HostColumn:
