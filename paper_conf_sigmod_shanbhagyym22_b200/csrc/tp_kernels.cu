@@ -133,7 +133,7 @@ __device__ __forceinline__ void decode_dfor(const Params& P, const Col& c, const
 // LoadRBitPack analogue: the 4 steps of [18] (2 scatters + 2 scans),
 // done per 512-row block by one warp, both blocks of the warp's round in turn:
 //  1. unpack: lane t takes the C consecutive entries [C t, C t + C) of both streams
-//     (C = 4 / 8 / 16 by the block's run count r, so one pass covers the block and a lane's
+//     (C = 1 / 2 / 4 / 8 / 16 by the block's run count r, so one pass covers the block and a lane's
 //     entries sit inside one 32-entry miniblock: one bitwidth and base per lane);
 //  2. run starts S = exclusive scan of the run lengths (lane-local scan + one warp scan);
 //  3. scatter: value V_e -> A[S_e], a start flag byte -> F[S_e] (plain stores: the starts
@@ -209,6 +209,10 @@ __device__ __forceinline__ void rfor_scatter(const uint32_t* bV, const uint32_t*
 }
 
 // steps 1-3 for both row blocks of the warp's round (block h -> scratch + h * RFOR_BLOCK_WORDS)
+// SMALLC: also the C = 1 / 2 bodies for blocks of few (long) runs -- single-column decodes
+// only: the query kernels keep the smaller code (their RFOR columns have short runs, and the
+// extra bodies cost the star kernels ~4 % through instruction-cache misses, measured)
+template <bool SMALLC = false>
 __device__ __forceinline__ void rfor_scatter_round(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                                    uint32_t* scratch) {
   const StreamView vv = stream_view(P, c.s0, C), vl = stream_view(P, c.s1, C);
@@ -225,7 +229,10 @@ __device__ __forceinline__ void rfor_scatter_round(const Params& P, const Col& c
     const uint32_t* bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
     const uint32_t* bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
     const uint32_t r = min(bV[0], 512u);  // run / value count
-    if (r <= 128u) rfor_scatter<4>(bV, bL, r, lane, A, F);
+    // C = entries per lane: the fewest that cover the block's runs (long runs: one entry per lane)
+    if (SMALLC && r <= 32u) rfor_scatter<1>(bV, bL, r, lane, A, F);
+    else if (SMALLC && r <= 64u) rfor_scatter<2>(bV, bL, r, lane, A, F);
+    else if (r <= 128u) rfor_scatter<4>(bV, bL, r, lane, A, F);
     else if (r <= 256u) rfor_scatter<8>(bV, bL, r, lane, A, F);
     else rfor_scatter<16>(bV, bL, r, lane, A, F);
   }
@@ -286,9 +293,10 @@ __device__ __forceinline__ uint32_t rfor_row(const RforChunk& k, uint32_t carry,
   return mm ? k.A[rfor_a_pos(32u * k.j + 31u - __clz(mm))] : carry;
 }
 
+template <bool SMALLC>
 __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                             uint32_t* scratch, uint32_t (&val)[32]) {
-  rfor_scatter_round(P, c, C, g, scratch);
+  rfor_scatter_round<SMALLC>(P, c, C, g, scratch);
   const RforChunk k = rfor_chunk(scratch, g.lane);
   rfor_fill(k, rfor_carry(k), val);
 }
@@ -331,7 +339,7 @@ __device__ __forceinline__ void decode_col(const Params& P, uint32_t ci, const S
   if ((MASK & M_NONE) && c.scheme == S_NONE) decode_none(P, c, C, g, val);
   else if ((MASK & M_FOR) && c.scheme == S_FOR) decode_for<COMPACT>(P, c, C, g, val);
   else if ((MASK & M_DFOR) && c.scheme == S_DFOR) decode_dfor<COMPACT>(P, c, C, g, val);
-  else if (MASK & M_RFOR) decode_rfor(P, c, C, g, scratch, val);
+  else if (MASK & M_RFOR) decode_rfor<!COMPACT>(P, c, C, g, scratch, val);
 }
 
 // ------------------------------------------------------------------ the pipeline

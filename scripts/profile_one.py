@@ -2,6 +2,7 @@
 """Run ONE decode of a bench_suite configuration (for ncu: capture the last launch).
 
   ncu --set full -k regex:k_decode -s 2 -c 1 -o out python scripts/profile_one.py for_b4 sum
+  modes: sum | global | enc (tp_gpu_encode of the column)
 """
 import os
 import sys
@@ -24,6 +25,12 @@ def main():
     print(name, "compressed bytes", h.nbytes(), "rows", rows, flush=True)
     acc = torch.zeros(1, dtype=torch.int64, device="cuda")
     out = torch.empty(rows, dtype=torch.int32, device="cuda") if mode == "global" else None
+    if mode == "enc":  # the GPU encoder on the same column
+        xd = torch.from_numpy(x).cuda()
+        for _ in range(3):
+            tp.gpu_encode(xd, cfg[1])
+        torch.cuda.synchronize()
+        return
     for _ in range(3):
         if mode == "sum":
             tp.tp_decode_sum(d.col, acc)
