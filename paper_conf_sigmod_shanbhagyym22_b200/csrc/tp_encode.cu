@@ -37,38 +37,54 @@ extern std::atomic<uint64_t> g_launches;
 namespace tp {
 namespace enc {
 
-constexpr int EW = 8;                                  // warps per CTA = tiles per chunk
+constexpr int EW = 8;                                  // warps per CTA
 constexpr int ETHREADS = 32 * EW;
-constexpr uint32_t CHUNK_ROWS = EW * TILE_ROWS;        // 4096 rows per chunk
 constexpr uint64_t ST_AGG = 1ull << 62, ST_INC = 2ull << 62, ST_VAL = (1ull << 62) - 1;
 constexpr int MODE_SIZES = 0;                          // SCHEME template value: all three plans, counts only
+
+// tiles per warp: FOR / DFOR -- 2 (lane l owns miniblock l & 15 of tile l >> 4, the decoder's
+// mapping); RFOR and the sizes pass -- 1 (the run scan takes the whole warp; for packing, lanes
+// 0-15 own the value stream's miniblocks and lanes 16-31 the run-length stream's)
+__host__ __device__ constexpr int tpw_of(int scheme) { return scheme == TP_FOR || scheme == TP_DFOR ? 2 : 1; }
+// sub-rounds per chunk: FOR / DFOR warps stage and pack 2 x 2 tiles before the chunk's
+// look-back (halves the look-back waits per row, measured); RFOR packs from registers after it
+__host__ __device__ constexpr int ks_of(int scheme) { return tpw_of(scheme) == 2 ? 2 : 1; }
+__host__ __device__ constexpr uint32_t chunk_rows(int scheme) {
+  return EW * tpw_of(scheme) * ks_of(scheme) * TILE_ROWS;
+}
+// per-warp shared words: FOR / DFOR per sub-round the two staged tiles, re-used in place as
+// the output staging (2 x 528 >= 2 x (1 + 4 (2 + 128)) words) + 16 relative block starts;
+// RFOR / sizes: X, run starts S, V, L
+__host__ __device__ constexpr uint32_t warp_words(int scheme) {
+  return tpw_of(scheme) == 2 ? 1056u * ks_of(scheme) + 16u : 2048u;
+}
+constexpr uint32_t STG_TILE = 528;
 
 // workspace (u64 words): [0] chunk counter, [1..2] stream totals, [3..4] max tile words,
 // [5] overflow flag, [6..9] sizes mode: FOR, DFOR, RFOR values, RFOR lengths; then the
 // look-back status words, two per chunk (stream 0, stream 1)
 constexpr int W_CTR = 0, W_TOT = 1, W_MTW = 3, W_OVF = 5, W_SIZES = 6, W_STATUS = 16;
 
-// per-warp plan of one stream of the current tile
-struct Plan {
-  int32_t ref[4];     // FOR / DFOR: per block; RFOR: [0]
-  uint32_t b[16];     // bitwidth of each miniblock (0 for absent ones)
-  uint32_t off[17];   // exclusive prefix of the miniblocks' data words; off[16] = total
-  uint32_t cnt[16];   // entries per miniblock (RFOR; FOR / DFOR: valid entries)
-  uint32_t words;     // the tile's words in this stream
-};
-struct WarpHdr {
-  Plan p[2];
-  uint32_t r;         // RFOR run count
-  uint32_t m;         // rows of the tile
-};
-// per-warp arrays (words): X (values), then DFOR deltas / RFOR V, S, L
-template <int SCHEME>
-__host__ __device__ constexpr int n_arrays() { return SCHEME == TP_FOR ? 1 : SCHEME == TP_DFOR ? 2 : 4; }
-constexpr uint32_t HDR_WORDS = (sizeof(WarpHdr) + 15) / 16 * 4;
-
 __device__ __forceinline__ uint32_t bitlen(uint32_t u) { return u ? 32u - __clz(u) : 0u; }
 
-// exclusive prefix of x over lanes 0..15 (lanes 16..31 get garbage); total in *tot
+// shared layout of staged rows: miniblock-major (32 words per 32-row miniblock), the 16-byte
+// chunk q of miniblock mb at chunk q ^ (mb & 7), so that 8 lanes reading chunk q of 8
+// consecutive miniblocks hit 8 distinct bank groups (conflict-free 128-bit loads)
+__device__ __forceinline__ uint32_t xs(uint32_t r) {
+  const uint32_t mb = r >> 5;
+  return (mb << 5) | ((((r >> 2) & 7u) ^ (mb & 7u)) << 2) | (r & 3u);
+}
+__device__ __forceinline__ void load_mb(const uint32_t* X, uint32_t mb, uint32_t (&v)[32]) {
+  const uint32_t* b = X + 32u * mb;
+  const uint32_t sw = mb & 7u;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const uint4 t = *reinterpret_cast<const uint4*>(b + 4u * ((uint32_t)q ^ sw));
+    v[4 * q] = t.x; v[4 * q + 1] = t.y; v[4 * q + 2] = t.z; v[4 * q + 3] = t.w;
+  }
+}
+
+// segmented (16-lane) exclusive prefix of x; *tot = the segment's total
 __device__ __forceinline__ uint32_t excl16(uint32_t x, uint32_t lane, uint32_t* tot) {
   uint32_t s = x;
 #pragma unroll
@@ -76,170 +92,130 @@ __device__ __forceinline__ uint32_t excl16(uint32_t x, uint32_t lane, uint32_t* 
     const uint32_t y = __shfl_up_sync(FULL, s, d);
     if ((lane & 15u) >= (uint32_t)d) s += y;
   }
-  *tot = __shfl_sync(FULL, s, 15);
+  *tot = __shfl_sync(FULL, s, (lane & 16u) | 15u);
   return s - x;
 }
+// bitwidth word of the 4 miniblocks j .. j+3 (R2), valid in lanes with j % 4 == 0
+__device__ __forceinline__ uint32_t bw_word(uint32_t b, uint32_t lane) {
+  const uint32_t b1 = __shfl_down_sync(FULL, b, 1), b2 = __shfl_down_sync(FULL, b, 2),
+                 b3 = __shfl_down_sync(FULL, b, 3);
+  return b | b1 << 8 | b2 << 16 | b3 << 24;
+}
 
-// FOR-plan the nblk blocks of 128 slots of src (slots >= nvalid are neutral pads, R8 / R13)
-__device__ void plan_for_blocks(const int32_t* src, uint32_t nvalid, uint32_t nblk, Plan& P, uint32_t lane,
-                                uint32_t extra_words) {
-#pragma unroll 1
-  for (uint32_t k = 0; k < nblk; ++k) {
-    const uint32_t s0 = 128u * k + 4u * lane;
-    const int4 q = *reinterpret_cast<const int4*>(src + s0);
-    const int32_t v[4] = {q.x, q.y, q.z, q.w};
-    int32_t mn = INT_MAX;
+// ---- bit packing of one 32-entry miniblock at compile-time bitwidth B (the inverse of
+// Alg. 1 lines 12-17: entry i at stream bits [i B, i B + B), LSB-first, R1); stores words
+// [0, nw) of the packed miniblock (nw = B for FOR, ceil(cnt B / 32) for the tight RFOR
+// miniblocks, R17).  Entries must already be < 2^B.
+template <int B>
+__device__ __forceinline__ void pack_fixed(const uint32_t (&u)[32], uint32_t* dst, uint32_t nw) {
+  if constexpr (B > 0) {
 #pragma unroll
-    for (int j = 0; j < 4; ++j)
-      if (s0 + j < nvalid) mn = min(mn, v[j]);
-    mn = __reduce_min_sync(FULL, mn);
-    const int32_t ref = 128u * k < nvalid ? mn : 0;  // a block of pads only: ref 0 (R14)
-    uint32_t o = 0u;
+    for (int k = 0; k < B; ++k) {
+      uint32_t w = 0u;
 #pragma unroll
-    for (int j = 0; j < 4; ++j)
-      if (s0 + j < nvalid) o |= (uint32_t)v[j] - (uint32_t)ref;  // offsets mod 2^32 (R4)
-    o |= __shfl_xor_sync(FULL, o, 1);
-    o |= __shfl_xor_sync(FULL, o, 2);
-    o |= __shfl_xor_sync(FULL, o, 4);
-    if ((lane & 7u) == 0) {
-      const uint32_t j = 4u * k + (lane >> 3);
-      P.b[j] = bitlen(o);  // bit length of the OR == bit length of the max (R3)
-      const uint32_t lo = 32u * j;
-      P.cnt[j] = nvalid > lo ? min(32u, nvalid - lo) : 0u;
+      for (int i = 0; i < 32; ++i) {
+        const int p = i * B - 32 * k;
+        if (p > -B && p < 32) w |= p >= 0 ? (u[i] << p) : (u[i] >> (-p));
+      }
+      if ((uint32_t)k < nw) dst[k] = w;
     }
-    if (lane == 0) P.ref[k] = ref;
   }
-  __syncwarp();
-  const uint32_t bj = lane < 16 && (lane >> 2) < nblk ? P.b[lane] : 0u;
-  uint32_t tot;
-  const uint32_t ex = excl16(bj, lane, &tot);  // full miniblocks: b words each
-  if (lane < 16) {
-    P.off[lane] = ex;
-    if (lane >= 4 * nblk) { P.b[lane] = 0u; P.cnt[lane] = 0u; }
-  }
-  if (lane == 0) {
-    P.off[16] = tot;
-    P.words = extra_words + 2u * nblk + tot;
-  }
-  __syncwarp();
 }
+#define TP_PCASE(B) \
+  case B:           \
+    pack_fixed<B>(u, dst, nw); break;
+// warp-cooperative dispatch: the specialised routine runs once per distinct bitwidth among
+// the lanes (as the decoder's unpack_mb)
+__device__ __forceinline__ void pack_mb(const uint32_t (&u)[32], uint32_t b, uint32_t* dst, uint32_t nw) {
+  uint32_t todo = FULL;
+  do {
+    const uint32_t bl = __shfl_sync(FULL, b, __ffs(todo) - 1);
+    const bool mine = b == bl;
+    todo &= ~__ballot_sync(FULL, mine);
+    if (mine) {
+      switch (bl) {
+        TP_PCASE(0) TP_PCASE(1) TP_PCASE(2) TP_PCASE(3) TP_PCASE(4) TP_PCASE(5) TP_PCASE(6) TP_PCASE(7)
+        TP_PCASE(8) TP_PCASE(9) TP_PCASE(10) TP_PCASE(11) TP_PCASE(12) TP_PCASE(13) TP_PCASE(14) TP_PCASE(15)
+        TP_PCASE(16) TP_PCASE(17) TP_PCASE(18) TP_PCASE(19) TP_PCASE(20) TP_PCASE(21) TP_PCASE(22) TP_PCASE(23)
+        TP_PCASE(24) TP_PCASE(25) TP_PCASE(26) TP_PCASE(27) TP_PCASE(28) TP_PCASE(29) TP_PCASE(30) TP_PCASE(31)
+        default: pack_fixed<32>(u, dst, nw); break;
+      }
+    }
+  } while (todo);
+}
+#undef TP_PCASE
 
-// FOR-plan one RFOR stream block of r entries (16 tight miniblocks of 32, R17)
-__device__ void plan_rfor_stream(const int32_t* src, uint32_t r, Plan& P, uint32_t lane) {
+// ---- FOR plan of the lane's miniblock j of a tile whose slots >= nvalid are neutral pads
+// (R8 / R13): block reference = signed min over the block's real slots (R4; 0 for a block of
+// pads only, R14), bitwidth = bit length of the OR of the offsets (== of the max, R3).
+// v: the slots; on return u = offsets (pads 0), b = bitwidth, ref = the block's reference.
+__device__ __forceinline__ void plan_for_mb(const uint32_t (&v)[32], uint32_t j, uint32_t nvalid,
+                                            uint32_t (&u)[32], uint32_t& b, int32_t& ref) {
+  const uint32_t lo = 32u * j;
+  const uint32_t cnt = nvalid > lo ? min(32u, nvalid - lo) : 0u;
   int32_t mn = INT_MAX;
-  for (uint32_t i = lane; i < r; i += 32) mn = min(mn, src[i]);
-  mn = __reduce_min_sync(FULL, mn);
-  const int32_t ref = mn;
-  uint32_t my_b = 0u;
-#pragma unroll 1
-  for (uint32_t q = 0; q < 16; ++q) {
-    if (32u * q >= r) break;  // warp-uniform
-    const uint32_t i = 32u * q + lane;
-    const uint32_t u = i < r ? (uint32_t)src[i] - (uint32_t)ref : 0u;
-    const uint32_t o = __reduce_or_sync(FULL, u);
-    if (lane == q) my_b = bitlen(o);
+#pragma unroll
+  for (int i = 0; i < 32; ++i)
+    if ((uint32_t)i < cnt) mn = min(mn, (int32_t)v[i]);
+  mn = min(mn, __shfl_xor_sync(FULL, mn, 1));
+  mn = min(mn, __shfl_xor_sync(FULL, mn, 2));
+  ref = 128u * (j >> 2) < nvalid ? mn : 0;
+  uint32_t o = 0u;
+#pragma unroll
+  for (int i = 0; i < 32; ++i) {
+    u[i] = (uint32_t)i < cnt ? v[i] - (uint32_t)ref : 0u;  // mod 2^32 (R4)
+    o |= u[i];
   }
-  const uint32_t cnt = lane < 16 ? (r > 32u * lane ? min(32u, r - 32u * lane) : 0u) : 0u;
-  const uint32_t wq = (cnt * my_b + 31u) >> 5;  // tight: ceil(cnt * b / 32) words
-  uint32_t tot;
-  const uint32_t ex = excl16(wq, lane, &tot);
-  if (lane < 16) {
-    P.b[lane] = my_b;
-    P.cnt[lane] = cnt;
-    P.off[lane] = ex;
-  }
-  if (lane == 0) {
-    P.ref[0] = ref;
-    P.off[16] = tot;
-    P.words = 6u + tot;
-  }
-  __syncwarp();
+  b = bitlen(o);
 }
 
-// runs of the tile (R18): V[idx] = value, S[idx] = start row, L[idx] = length; returns r
-__device__ uint32_t find_runs(const int32_t* X, uint32_t m, int32_t* V, int32_t* S, int32_t* L, uint32_t lane) {
+// runs of one 512-row tile (R18; X staged with xs): V[xs(e)] = value of run e, L[xs(e)] =
+// its length; returns r.  S = scratch (run start rows).
+__device__ uint32_t find_runs(const uint32_t* X, uint32_t m, uint32_t* V, uint32_t* S, uint32_t* L,
+                              uint32_t lane) {
   uint32_t base = 0u;
   const uint32_t lt = (1u << lane) - 1u;
 #pragma unroll 1
   for (uint32_t q = 0; q < 16; ++q) {
-    if (32u * q >= m) break;
+    if (32u * q >= m) break;  // warp-uniform
     const uint32_t row = 32u * q + lane;
-    const bool f = row < m && (row == 0 || X[row] != X[row - 1]);
+    const uint32_t xv = X[xs(row)];
+    const bool f = row < m && (row == 0 || xv != X[xs(row - 1)]);
     const uint32_t bal = __ballot_sync(FULL, f);
     if (f) {
-      const uint32_t idx = base + __popc(bal & lt);
-      V[idx] = X[row];
-      S[idx] = (int32_t)row;
+      const uint32_t e = base + __popc(bal & lt);
+      V[xs(e)] = xv;
+      S[e] = row;
     }
     base += __popc(bal);
   }
   __syncwarp();
-  for (uint32_t i = lane; i < base; i += 32) L[i] = (i + 1 < base ? S[i + 1] : (int32_t)m) - S[i];
+  for (uint32_t e = lane; e < base; e += 32) L[xs(e)] = (e + 1 < base ? S[e + 1] : m) - S[e];
   __syncwarp();
   return base;
 }
 
-// output word w of miniblock j (entries src[0..cnt), bitwidth b, reference ref): the OR of
-// every entry whose bit range [i b, i b + b) meets [32 w, 32 w + 32) (R1)
-__device__ __forceinline__ uint32_t pack_word(const int32_t* src, uint32_t cnt, uint32_t b, uint32_t w,
-                                              int32_t ref) {
-  const uint32_t bit0 = 32u * w;
-  uint32_t i = bit0 / b;
-  const uint32_t iend = min(cnt, (bit0 + 31u) / b + 1u);
-  uint32_t word = 0u;
-  for (; i < iend; ++i) {
-    const uint32_t u = (uint32_t)src[i] - (uint32_t)ref;
-    const int p = (int)(i * b) - (int)bit0;
-    word |= p >= 0 ? (u << p) : (u >> (-p));
-  }
-  return word;
-}
-
-// last miniblock j with off[j] <= t (t < off[16]): its data holds word t
-__device__ __forceinline__ uint32_t find_mb(const uint32_t* off, uint32_t t) {
-  uint32_t lo = 0;
+// RFOR plan of the lane's miniblock j (16 tight miniblocks of 32 entries, R17) of the stream
+// whose entries sit in A (xs layout), r entries
+__device__ __forceinline__ void plan_rfor_mb(const uint32_t* A, uint32_t j, uint32_t r, uint32_t (&u)[32],
+                                             uint32_t& b, int32_t& ref, uint32_t& cnt) {
+  uint32_t v[32];
+  load_mb(A, j, v);
+  cnt = r > 32u * j ? min(32u, r - 32u * j) : 0u;
+  int32_t mn = INT_MAX;
 #pragma unroll
-  for (uint32_t step = 8; step > 0; step >>= 1)
-    if (off[lo + step] <= t) lo += step;
-  return lo;
-}
-
-// write one tile's FOR / DFOR blocks (data base B, first block index blk0)
-__device__ void write_for_tile(const int32_t* src, const Plan& P, uint32_t nblk, bool dfor, int32_t first,
-                               uint64_t B, uint64_t blk0, uint32_t* starts, uint32_t* data, uint32_t lane) {
-  const uint64_t d0 = B + (dfor ? 1u : 0u);
-  if (dfor && lane == 0) data[B] = (uint32_t)first;  // first value of the tile
-  if (lane < nblk) {
-    const uint64_t bs = d0 + 2u * lane + P.off[4 * lane];
-    starts[blk0 + lane] = (uint32_t)bs;
-    data[bs] = (uint32_t)P.ref[lane];
-    data[bs + 1] = P.b[4 * lane] | P.b[4 * lane + 1] << 8 | P.b[4 * lane + 2] << 16 | P.b[4 * lane + 3] << 24;
+  for (int i = 0; i < 32; ++i)
+    if ((uint32_t)i < cnt) mn = min(mn, (int32_t)v[i]);
+#pragma unroll
+  for (int d = 1; d < 16; d <<= 1) mn = min(mn, __shfl_xor_sync(FULL, mn, d));
+  ref = mn;
+  uint32_t o = 0u;
+#pragma unroll
+  for (int i = 0; i < 32; ++i) {
+    u[i] = (uint32_t)i < cnt ? v[i] - (uint32_t)ref : 0u;
+    o |= u[i];
   }
-  const uint32_t tot = P.off[16];
-  for (uint32_t t = lane; t < tot; t += 32) {
-    const uint32_t j = find_mb(P.off, t);
-    const uint32_t k = j >> 2;
-    data[d0 + 2u * (k + 1u) + t] = pack_word(src + 32u * j, P.cnt[j], P.b[j], t - P.off[j], P.ref[k]);
-  }
-}
-
-// write one RFOR stream block at B
-__device__ void write_rfor_stream(const int32_t* src, const Plan& P, uint32_t r, uint64_t B, uint64_t blk,
-                                  uint32_t* starts, uint32_t* data, uint32_t lane) {
-  if (lane == 0) {
-    starts[blk] = (uint32_t)B;
-    data[B] = r;
-    data[B + 1] = (uint32_t)P.ref[0];
-  }
-  if (lane >= 2 && lane < 6) {
-    const uint32_t q = lane - 2;
-    data[B + lane] = P.b[4 * q] | P.b[4 * q + 1] << 8 | P.b[4 * q + 2] << 16 | P.b[4 * q + 3] << 24;
-  }
-  const uint32_t tot = P.off[16];
-  for (uint32_t t = lane; t < tot; t += 32) {
-    const uint32_t j = find_mb(P.off, t);
-    data[B + 6u + t] = pack_word(src + 32u * j, P.cnt[j], P.b[j], t - P.off[j], P.ref[0]);
-  }
+  b = bitlen(o);
 }
 
 // ---- decoupled look-back (stream s): exclusive prefix of chunk c's words
@@ -285,7 +261,7 @@ __device__ uint64_t look_back(unsigned long long* status, uint32_t c, uint64_t a
 template <int SCHEME>
 struct EncArgs {
   const int32_t* x;
-  uint32_t n, ntiles, nchunks, nblocks;  // nblocks: block_starts entries - 1 (stream 0)
+  uint32_t n, ntiles, nchunks, nblocks;  // nblocks: block_starts entries - 1
   uint32_t* starts0;
   uint32_t* data0;
   uint32_t* starts1;
@@ -295,19 +271,21 @@ struct EncArgs {
 };
 
 template <int SCHEME>
-__global__ void __launch_bounds__(ETHREADS) k_encode(const __grid_constant__ EncArgs<SCHEME> A) {
+__global__ void __launch_bounds__(ETHREADS, 3) k_encode(const __grid_constant__ EncArgs<SCHEME> A) {
   extern __shared__ __align__(16) uint32_t esm[];
   constexpr bool SIZES = SCHEME == MODE_SIZES;
-  constexpr int NA = SIZES ? 4 : n_arrays<SCHEME>();
+  constexpr int TPW = tpw_of(SCHEME);   // tiles per warp and sub-round
+  constexpr int KS = ks_of(SCHEME);     // sub-rounds per chunk (staged side by side)
+  constexpr int TW = TPW * KS;          // tiles per warp and chunk
+  constexpr bool DF = SCHEME == TP_DFOR;
+  constexpr int NS = SCHEME == TP_RFOR ? 2 : 1;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
+  const uint32_t seg = lane >> 4, j = lane & 15u;
   __shared__ uint32_t s_chunk;
-  __shared__ uint32_t s_words[2][EW];
+  __shared__ uint32_t s_words[2][EW * 4];
   __shared__ unsigned long long s_base[2], s_agg[2];
-  WarpHdr& H = *reinterpret_cast<WarpHdr*>(esm + warp * (HDR_WORDS + NA * 512u));
-  int32_t* X = reinterpret_cast<int32_t*>(esm + warp * (HDR_WORDS + NA * 512u) + HDR_WORDS);
-  int32_t* A1 = X + 512;  // DFOR deltas / RFOR values
-  int32_t* A2 = X + 1024; // RFOR run starts
-  int32_t* A3 = X + 1536; // RFOR run lengths
+  uint32_t* Xw = esm + warp * warp_words(SCHEME);
+  uint32_t* bsr = Xw + KS * 1056u;  // FOR / DFOR: block starts relative to their tile, 4 per tile
   unsigned long long* work = A.work;
 
   while (true) {
@@ -315,73 +293,118 @@ __global__ void __launch_bounds__(ETHREADS) k_encode(const __grid_constant__ Enc
     __syncthreads();
     const uint32_t c = s_chunk;
     if (c >= A.nchunks) break;
-    const uint32_t t = c * EW + warp;  // this warp's tile
-    const bool has = t < A.ntiles;
-    const uint32_t r0 = t * TILE_ROWS;
-    const uint32_t m = has ? min((uint32_t)TILE_ROWS, A.n - r0) : 0u;
-    uint32_t w0 = 0u, w1 = 0u, wf = 0u, wd = 0u, wv = 0u, wl = 0u;
-    if (has) {
-      // ---- stage the tile (coalesced 16-byte loads; the tail row by row)
-      if (m == TILE_ROWS) {
+    const uint32_t t0 = (c * EW + warp) * TW;  // this warp's first tile
+    uint32_t u[32];
+    uint32_t b = 0u, P = 0u, nw = 0u;  // bitwidth, data-word offset, words of the lane's miniblock
+    int32_t ref = 0;
+    uint32_t wv = 0u, wl = 0u, r = 0u, my_t = t0;
+#pragma unroll 1
+    for (uint32_t p = 0; p < (uint32_t)KS; ++p) {
+      uint32_t* X = Xw + p * 1056u;
+      uint32_t* S = X + 512;  // RFOR / sizes: run starts, then V, L
+      uint32_t* V = X + 1024;
+      uint32_t* L = X + 1536;
+      const uint32_t tp0 = t0 + p * TPW;
+      const uint32_t r0 = tp0 * TILE_ROWS;
+      const uint32_t mrows = tp0 < A.ntiles ? min((uint32_t)(TPW * TILE_ROWS), A.n - r0) : 0u;
+      // ---- stage the tiles (coalesced 16-byte loads, miniblock-major swizzled rows)
+      if (mrows == TPW * TILE_ROWS) {
         const int4* src = reinterpret_cast<const int4*>(A.x + r0);
+        int4 q[4 * TPW];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          const int4 q = __ldcs(src + 32 * k + lane);
-          *reinterpret_cast<int4*>(X + 128 * k + 4 * lane) = q;
-        }
-      } else {
-        for (uint32_t i = lane; i < TILE_ROWS; i += 32) X[i] = i < m ? __ldcs(A.x + r0 + i) : 0;
+        for (int k = 0; k < 4 * TPW; ++k) q[k] = __ldcs(src + 32 * k + lane);
+#pragma unroll
+        for (int k = 0; k < 4 * TPW; ++k) *reinterpret_cast<int4*>(X + xs(128u * k + 4u * lane)) = q[k];
+      } else if (mrows > 0) {
+        for (uint32_t rr = lane; rr < TPW * TILE_ROWS; rr += 32)
+          X[xs(rr)] = rr < mrows ? (uint32_t)A.x[r0 + rr] : 0u;
       }
       __syncwarp();
+      // the lane's tile (FOR / DFOR: tile tp0 + seg; else tp0)
+      my_t = tp0 + (TPW == 2 ? seg : 0u);
+      const uint32_t m = my_t < A.ntiles ? min((uint32_t)TILE_ROWS, A.n - my_t * TILE_ROWS) : 0u;
       const uint32_t nblk = (m + 127u) >> 7;
-      if (SIZES || SCHEME == TP_FOR) {
-        plan_for_blocks(X, m, nblk, H.p[0], lane, 0u);
-        wf = H.p[0].words;
-      }
-      if (SIZES || SCHEME == TP_DFOR) {
-        for (uint32_t s = lane; s < TILE_ROWS; s += 32)  // delta slots (R12, R13)
-          A1[s] = s + 1 < m ? (int32_t)((uint32_t)X[s + 1] - (uint32_t)X[s]) : 0;
-        __syncwarp();
-        plan_for_blocks(A1, m - 1u, nblk, H.p[0], lane, 1u);
-        wd = H.p[0].words;
+      uint32_t tw = 0u, first = 0u, wf = 0u, wd = 0u;
+      if (SIZES || SCHEME == TP_FOR || SCHEME == TP_DFOR) {
+        uint32_t v[32];
+        load_mb(X, (TPW == 2 ? 16u * seg : 0u) + j, v);
+        first = v[0];
+        if (SIZES || SCHEME == TP_FOR) {
+          plan_for_mb(v, j, m, u, b, ref);
+          const uint32_t bj = (j >> 2) < nblk ? b : 0u;
+          uint32_t tot;
+          P = excl16(bj, lane, &tot);
+          nw = bj;
+          tw = 2u * nblk + tot;
+          wf = tw;
+        }
+        if (SIZES || SCHEME == TP_DFOR) {
+          // delta slots (R12, R13): slot s = x[s+1] - x[s] for s < m - 1, neutral pads after
+          const uint32_t nxt = __shfl_down_sync(FULL, v[0], 1);
+#pragma unroll
+          for (int i = 0; i < 31; ++i) v[i] = v[i + 1] - v[i];
+          v[31] = nxt - v[31];
+          plan_for_mb(v, j, m ? m - 1u : 0u, u, b, ref);
+          const uint32_t bj = (j >> 2) < nblk ? b : 0u;
+          uint32_t tot;
+          P = excl16(bj, lane, &tot);
+          nw = bj;
+          tw = m > 0 ? 1u + 2u * nblk + tot : 0u;  // first value + blocks (no tile: no words)
+          wd = tw;
+        }
+        if (!SIZES) {
+          __syncwarp();  // every lane holds its rows: the staged tiles become the output staging
+          uint32_t* stg = X + seg * STG_TILE;
+          const uint32_t blk = j >> 2, d0 = DF ? 1u : 0u;
+          const uint32_t bw = bw_word(b, lane);  // (warp-collective: outside the per-tile branch)
+          if (m > 0) {
+            if (DF && j == 0) stg[0] = first;  // first value of the tile
+            if ((j & 3u) == 0 && blk < nblk) {
+              const uint32_t bs = d0 + 2u * blk + P;  // header of block blk (P = its first mb's offset)
+              stg[bs] = (uint32_t)ref;
+              stg[bs + 1] = bw;
+              bsr[4u * (p * TPW + seg) + blk] = bs;
+            }
+          }
+          // one call site for every lane (warp-collective dispatch); nw = 0 past the column's end
+          pack_mb(u, nw, stg + d0 + 2u * (blk + 1u) + P, nw);
+          if (j == 0) s_words[0][TW * warp + p * TPW + seg] = tw;
+        }
       }
       if (SIZES || SCHEME == TP_RFOR) {
-        const uint32_t r = find_runs(X, m, A1, A2, A3, lane);
-        if (lane == 0) H.r = r;
-        plan_rfor_stream(A1, r, H.p[0], lane);
-        plan_rfor_stream(A3, r, H.p[1], lane);
-        wv = H.p[0].words;
-        wl = H.p[1].words;
+        uint32_t cnt = 0u;
+        if (m > 0) r = find_runs(X, m, V, S, L, lane);
+        plan_rfor_mb(seg ? L : V, j, r, u, b, ref, cnt);
+        nw = (cnt * b + 31u) >> 5;  // tight: ceil(cnt b / 32) words
+        uint32_t tot;
+        P = excl16(nw, lane, &tot);
+        tw = m > 0 ? 6u + tot : 0u;
+        wv = __shfl_sync(FULL, tw, 0);
+        wl = __shfl_sync(FULL, tw, 16);
+        if (!SIZES && lane == 0) { s_words[0][warp] = wv; s_words[1][warp] = wl; }
       }
-      w0 = SCHEME == TP_FOR ? wf : SCHEME == TP_DFOR ? wd : wv;
-      w1 = SCHEME == TP_RFOR ? wl : 0u;
-    }
-    if (SIZES) {
-      // counts only: one atomic per warp and scheme stream
-      if (lane == 0 && has) {
+      if (SIZES && lane == 0 && m > 0) {
         atomicAdd(work + W_SIZES + 0, (unsigned long long)wf);
         atomicAdd(work + W_SIZES + 1, (unsigned long long)wd);
         atomicAdd(work + W_SIZES + 2, (unsigned long long)wv);
         atomicAdd(work + W_SIZES + 3, (unsigned long long)wl);
       }
+    }
+    if (SIZES) {
       __syncthreads();
       continue;
     }
-    if (lane == 0) {
-      s_words[0][warp] = w0;
-      s_words[1][warp] = w1;
-    }
-    if (SCHEME != TP_RFOR && threadIdx.x == 0) s_base[1] = s_agg[1] = 0;
+    // ---- the chunk's offsets by look-back (warp s: stream s)
     __syncthreads();
-    // ---- chunk offsets: warp 0 (stream 0) and warp 1 (stream 1, RFOR) look back
-    constexpr int NS = SCHEME == TP_RFOR ? 2 : 1;
+    constexpr int NT = EW * TW;
     if (warp < NS) {
-      const uint32_t mine = lane < EW ? s_words[warp][lane] : 0u;
-      uint64_t agg = mine, mx = mine;
+      const uint32_t mine = lane < NT ? s_words[warp][lane] : 0u;
+      uint64_t agg = mine;
+      uint32_t mx = mine;
 #pragma unroll
       for (int d = 16; d > 0; d >>= 1) {
         agg += __shfl_xor_sync(FULL, agg, d);
-        mx = max(mx, (uint64_t)__shfl_xor_sync(FULL, (uint32_t)mx, d));
+        mx = max(mx, __shfl_xor_sync(FULL, mx, d));
       }
       const uint64_t base = look_back(work + W_STATUS + (uint64_t)warp * A.nchunks, c, agg, lane);
       if (lane == 0) {
@@ -393,26 +416,57 @@ __global__ void __launch_bounds__(ETHREADS) k_encode(const __grid_constant__ Enc
         if (c == A.nchunks - 1) work[W_TOT + warp] = base + agg;
       }
     }
+    if (SCHEME != TP_RFOR && threadIdx.x == 0) s_base[1] = s_agg[1] = 0;
     __syncthreads();
-    // ---- write: block_starts, headers, packed words
     const bool ovf = s_base[0] + s_agg[0] > A.cap0 || (SCHEME == TP_RFOR && s_base[1] + s_agg[1] > A.cap1);
-    if (has && !ovf) {
+    if (t0 < A.ntiles && !ovf) {
+      // the warp's base word in each stream: the chunk base + the earlier tiles of the chunk
       uint64_t B0 = s_base[0], B1 = s_base[1];
-      for (uint32_t w = 0; w < warp; ++w) {
-        B0 += s_words[0][w];
-        B1 += s_words[1][w];
-      }
-      const uint32_t nblk = (m + 127u) >> 7;
-      if (SCHEME == TP_FOR) {
-        write_for_tile(X, H.p[0], nblk, false, 0, B0, 4ull * t, A.starts0, A.data0, lane);
-      } else if (SCHEME == TP_DFOR) {
-        write_for_tile(A1, H.p[0], nblk, true, X[0], B0, 4ull * t, A.starts0, A.data0, lane);
+      for (uint32_t k = 0; k < TW * warp; ++k) B0 += s_words[0][k];
+      for (uint32_t k = 0; k < warp && SCHEME == TP_RFOR; ++k) B1 += s_words[1][k];
+      uint64_t e0 = B0, e1 = B1 + wl;  // end of the warp's words
+      if (SCHEME == TP_RFOR) {
+        // header [r][ref][4 bitwidth words] and the tight miniblocks, straight from registers
+        const uint64_t Bs = seg ? B1 : B0;
+        uint32_t* data = seg ? A.data1 : A.data0;
+        uint32_t* starts = seg ? A.starts1 : A.starts0;
+        const uint32_t bw = bw_word(b, lane);
+        if (j == 0) {
+          starts[my_t] = (uint32_t)Bs;
+          data[Bs] = r;
+          data[Bs + 1] = (uint32_t)ref;
+        }
+        if ((j & 3u) == 0) data[Bs + 2 + (j >> 2)] = bw;
+        pack_mb(u, b, data + Bs + 6 + P, nw);
+        e0 = B0 + wv;
       } else {
-        write_rfor_stream(A1, H.p[0], H.r, B0, t, A.starts0, A.data0, lane);
-        write_rfor_stream(A3, H.p[1], H.r, B1, t, A.starts1, A.data1, lane);
+        // block_starts (lane 4 tl + blk: block blk of the warp's tile tl), then the staged
+        // words of the warp's tiles, coalesced
+        uint64_t off = 0;
+        const uint32_t tl = lane >> 2, blk = lane & 3u;
+        uint64_t my_off = 0;
+#pragma unroll 1
+        for (uint32_t k = 0; k < (uint32_t)TW; ++k) {
+          if (k == tl) my_off = off;
+          off += s_words[0][TW * warp + k];
+        }
+        const uint32_t t = t0 + tl;
+        if (tl < (uint32_t)TW && t < A.ntiles) {
+          const uint32_t mt = min((uint32_t)TILE_ROWS, A.n - t * TILE_ROWS);
+          if (blk < ((mt + 127u) >> 7)) A.starts0[4ull * t + blk] = (uint32_t)(B0 + my_off + bsr[lane]);
+        }
+        uint64_t o = B0;
+#pragma unroll 1
+        for (uint32_t k = 0; k < (uint32_t)TW; ++k) {
+          const uint32_t wk = s_words[0][TW * warp + k];
+          const uint32_t* src = Xw + (k / TPW) * 1056u + (k % TPW) * STG_TILE;
+          for (uint32_t i = lane; i < wk; i += 32) A.data0[o + i] = src[i];
+          o += wk;
+        }
+        e0 = o;
       }
-      if (t == A.ntiles - 1) {  // the column's end: last block_starts entry + zero guards (R6, R9)
-        const uint64_t e0 = B0 + w0, e1 = B1 + w1;
+      // the column's end: last block_starts entry + zero guards (R6, R9)
+      if (t0 + TW >= A.ntiles) {
         if (lane < TP_GUARD_WORDS) {
           A.data0[e0 + lane] = 0u;
           A.starts0[A.nblocks + 1 + lane] = 0u;
@@ -456,12 +510,13 @@ static int enc_grid(K kernel, size_t smem) {
   return g_enc_sms * std::max(1, occ);
 }
 
-static uint64_t nchunks_of(uint64_t n) { return (n + CHUNK_ROWS - 1) / CHUNK_ROWS; }
+static uint64_t nchunks_of(uint64_t n, int scheme = MODE_SIZES) {
+  return (n + chunk_rows(scheme) - 1) / chunk_rows(scheme);
+}
 
 template <int SCHEME>
 static tp_status launch_encode(const EncArgs<SCHEME>& a, void* stream) {
-  constexpr int NA = SCHEME == MODE_SIZES ? 4 : n_arrays<SCHEME>();
-  const size_t smem = (size_t)EW * (HDR_WORDS + NA * 512u) * 4u;
+  const size_t smem = (size_t)EW * warp_words(SCHEME) * 4u;
   const int grid = std::max(1, std::min<int>(enc_grid(k_encode<SCHEME>, smem), (int)a.nchunks));
   k_encode<SCHEME><<<grid, ETHREADS, smem, (cudaStream_t)stream>>>(a);
   tp::g_launches.fetch_add(1, std::memory_order_relaxed);
@@ -571,7 +626,7 @@ tp_status tp_gpu_encode_launch(int scheme, const int32_t* d_x, uint64_t n, uint3
     a.x = d_x;
     a.n = (uint32_t)n;
     a.ntiles = (uint32_t)((n + TILE_ROWS - 1) / TILE_ROWS);
-    a.nchunks = (uint32_t)nchunks_of(n);
+    a.nchunks = (uint32_t)nchunks_of(n, scheme);
     a.nblocks = (uint32_t)nb;
     a.starts0 = d_starts0; a.data0 = d_data0; a.cap0 = cap0;
     a.starts1 = d_starts1; a.data1 = d_data1; a.cap1 = cap1;
