@@ -113,3 +113,18 @@ def mixed_columns(seed: int = 77):
         yield f"neg_n{n}", rng.integers(-(2**31), 2**31, n, dtype=np.int64).astype(np.int32)
         yield f"runs_n{n}", runs(n, 6, seed=int(rng.integers(1 << 30)))
         yield f"sorted_n{n}", np.sort(rng.integers(0, 1 << 20, n)).astype(np.int32)
+
+
+def bernoulli_bitmap(n: int, sigma: float, seed: int = 6000) -> np.ndarray:
+    """Predicate bitvector of the random-access experiment: each of the n rows
+    selected independently with probability sigma.  Returned as little-endian u32 words,
+    bit i of word k = row 32 k + i (include/tilepack.h tp_bitmap_sum), ceil(n/32) words."""
+    rng = np.random.default_rng(seed)
+    words = (n + 31) // 32
+    bits = np.zeros(words * 32, np.uint8)
+    if sigma >= 1.0:
+        bits[:n] = 1
+    elif sigma > 0.0:
+        k = rng.binomial(n, sigma)
+        bits[rng.choice(n, size=k, replace=False) if k < n // 4 else np.flatnonzero(rng.random(n) < sigma)] = 1
+    return np.packbits(bits, bitorder="little").view(np.uint32).copy()

@@ -209,6 +209,16 @@ typedef struct {
 tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int ncols, int agg,
                         int64_t* d_sums, uint64_t* d_counts, uint32_t ngroups, void* stream);
 
+/* Random access under a predicate bitvector:
+ *   *d_sum += sum of x[i] over the rows i whose bit is set,
+ * bit i of the bitvector = bit (i mod 32) of DEVICE word d_bitmap[i / 32] (LSB-first; at least
+ * ceil(n / 32) words; bits past n are ignored).  A 512-row tile whose bits are all zero is
+ * skipped without reading any of its compressed words; GPU-FOR and None also skip every
+ * 32-row miniblock whose bitvector word is zero (a FOR miniblock is read through its block
+ * header, Alg. 1), GPU-DFOR / GPU-RFOR decode each selected tile whole.  Any scheme, one
+ * kernel, asynchronous on `stream`. */
+tp_status tp_bitmap_sum(const tp_column* dcol, const uint32_t* d_bitmap, int64_t* d_sum, void* stream);
+
 /* The uncompressed baseline "None": *d_sum += sum of the n int32
  * values of DEVICE array d_x (16-byte aligned), 128-bit streaming loads.
  * Used as the measured HBM read roof of the same consumer. */

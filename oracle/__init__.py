@@ -228,6 +228,15 @@ def select_project_sum(cols, lo, hi, proj: str = "col", a: int = 0, b: int = 0) 
     return int(lib().orc_select_project_sum(ptrs, len(cols), _p(lo), _p(hi), n, PROJ[proj], a, b))
 
 
+def bitmap_sum(x, bitmap) -> int:
+    """Random access under a predicate bitvector, by its plain definition:
+    the int64 sum of x[i] over rows i whose bit is set (bit i = bit i % 32 of word i // 32)."""
+    x = _col(x)
+    n = len(x)
+    bits = np.unpackbits(np.ascontiguousarray(bitmap, np.uint32).view(np.uint8), bitorder="little")[:n]
+    return int(x[bits.astype(bool)].astype(np.int64).sum())
+
+
 def column_sum(x) -> int:
     x = _col(x)
     return int(lib().orc_sum(_p(x), len(x)))

@@ -1061,6 +1061,130 @@ __global__ void __launch_bounds__(THREADS, TP_QUERY_MINB)
   run_pipeline(P, op);
 }
 
+
+// ------------------------------------------------------------------ random access (bitvector)
+// a predicate bitvector selects rows; a compressed tile whose 512 bits are all
+// zero is skipped entirely (no block_starts, header or data read), otherwise it is decoded
+// and the bitvector applied.  Here the skip goes further for GPU-FOR and None: a 32-row
+// miniblock whose bitvector word is zero is not read either (FOR reads the block header and
+// the miniblock's b words, None its one 128-byte line); GPU-DFOR / GPU-RFOR
+// decode the whole tile (the prefix sum / run expansion needs every earlier entry).
+// One warp per pair of tiles, lane = miniblock (the pipeline's mapping), straight from
+// global memory (L1-cached loads; no staging: the access pattern is data-dependent).
+template <uint32_t MASK>
+__global__ void __launch_bounds__(256) k_bitmap_sum(const __grid_constant__ Params P, const uint32_t* __restrict__ bm,
+                                                    unsigned long long* out) {
+  extern __shared__ __align__(16) uint32_t rsm[];
+  const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+  const uint32_t seg = lane >> 4, j = lane & 15u;
+  const Col& c = P.col[0];
+  const Stream& st = P.st[c.s0];
+  uint32_t* scratch = rsm + warp * RFOR_SCRATCH_WORDS;
+  const uint32_t npairs = (P.ntiles + 1u) >> 1;
+  const uint32_t nmb = (P.n + 31u) >> 5;
+  uint64_t acc = 0;
+  for (uint32_t pair = blockIdx.x * (blockDim.x >> 5) + warp; pair < npairs; pair += gridDim.x * (blockDim.x >> 5)) {
+    const uint32_t t = 2u * pair + seg;
+    const uint32_t mb = 16u * t + j;
+    uint32_t w = 0u;
+    if (mb < nmb) {
+      w = __ldg(bm + mb);
+      const uint32_t rows = P.n - 32u * mb;
+      if (rows < 32u) w &= (1u << rows) - 1u;  // bits past the column's end
+    }
+    const uint32_t any = __ballot_sync(FULL, w != 0u);
+    if (any == 0u) continue;  // both tiles unselected: skipped without a read
+    const bool tile_any = ((any >> (16u * seg)) & 0xffffu) != 0u;
+    if ((MASK & M_NONE) && c.scheme == S_NONE) {
+      if (w) {  // one 128-byte line per selected miniblock
+        const uint4* line = reinterpret_cast<const uint4*>(st.data + 32u * mb);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+          const uint4 a = __ldg(line + q);
+          const uint32_t v4[4] = {a.x, a.y, a.z, a.w};
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            if ((w >> (4 * q + k)) & 1u) acc += (uint64_t)(int64_t)(int32_t)v4[k];
+        }
+      }
+    } else if ((MASK & M_FOR) && c.scheme == S_FOR) {
+      // Alg. 1 for the selected miniblocks only: block_starts -> header -> the b words (the
+      // bitwidth-specialised unpack, warp-collective: unselected lanes take b = 0)
+      uint32_t ref = 0u, b = 0u;
+      const uint32_t* mw = st.data;
+      if (w) {
+        const uint32_t s = __ldg(st.starts + (mb >> 2));
+        ref = __ldg(st.data + s);
+        const uint32_t bw = __ldg(st.data + s + 1);
+        b = min((bw >> (8u * (mb & 3u))) & 255u, 32u);
+        mw = st.data + s + 2 + bw_prefix(bw, mb & 3u);
+      }
+      uint32_t e[32];
+      unpack_mb(mw, b, e);
+#pragma unroll
+      for (int i = 0; i < 32; ++i)
+        if ((w >> i) & 1u) acc += (uint64_t)(int64_t)(int32_t)(ref + e[i]);
+    } else if ((MASK & M_DFOR) && c.scheme == S_DFOR) {
+      // the whole tile: deltas of every miniblock, exclusive prefix inside the tile (R13)
+      uint32_t run = 0u, first = 0u, ref = 0u, b = 0u;
+      const uint32_t* mw = st.data;
+      const bool live = tile_any && (mb >> 2) < c.nblocks;
+      if (live) {
+        const uint32_t s = __ldg(st.starts + (mb >> 2));
+        first = __ldg(st.data + __ldg(st.starts + 4u * t) - 1u);
+        ref = __ldg(st.data + s);
+        const uint32_t bw = __ldg(st.data + s + 1);
+        b = min((bw >> (8u * (mb & 3u))) & 255u, 32u);
+        mw = st.data + s + 2 + bw_prefix(bw, mb & 3u);
+      }
+      uint32_t e[32];
+      unpack_mb(mw, b, e);  // b = 0 (all zero) for lanes outside a selected tile
+      uint32_t val[32];
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        val[i] = run;
+        run += ref + e[i];
+      }
+      const uint32_t incl = seg16_inclusive_scan(run);
+      const uint32_t base = first + (incl - run);
+#pragma unroll
+      for (int i = 0; i < 32; ++i)
+        if ((w >> i) & 1u) acc += (uint64_t)(int64_t)(int32_t)(val[i] + base);
+    } else if (MASK & M_RFOR) {
+      // the whole tile: value / run-length streams scattered and expanded (steps 1-4 of
+      // decode_rfor, reading the stream blocks from global memory)
+      const Stream& sl = P.st[c.s1];
+      __syncwarp();
+#pragma unroll 1
+      for (uint32_t h = 0; h < 2; ++h) {
+        uint32_t* A = scratch + h * RFOR_BLOCK_WORDS;
+        uint8_t* F = reinterpret_cast<uint8_t*>(A + RFOR_A_WORDS);
+        st_shared_v4(reinterpret_cast<uint32_t*>(F) + 4u * lane, 0u, 0u, 0u, 0u);
+        __syncwarp();
+        const uint32_t th = 2u * pair + h;
+        if (th >= P.ntiles || !((any >> (16u * h)) & 0xffffu)) continue;  // warp-uniform
+        const uint32_t* bV = st.data + __ldg(st.starts + th);
+        const uint32_t* bL = sl.data + __ldg(sl.starts + th);
+        const uint32_t r = min(__ldg(bV), 512u);
+        if (r <= 32u) rfor_scatter<1>(bV, bL, r, lane, A, F);
+        else if (r <= 64u) rfor_scatter<2>(bV, bL, r, lane, A, F);
+        else if (r <= 128u) rfor_scatter<4>(bV, bL, r, lane, A, F);
+        else if (r <= 256u) rfor_scatter<8>(bV, bL, r, lane, A, F);
+        else rfor_scatter<16>(bV, bL, r, lane, A, F);
+      }
+      __syncwarp();
+      const RforChunk k = rfor_chunk(scratch, lane);
+      uint32_t val[32];
+      rfor_fill(k, rfor_carry(k), val);
+#pragma unroll
+      for (int i = 0; i < 32; ++i)
+        if ((w >> i) & 1u) acc += (uint64_t)(int64_t)(int32_t)val[i];
+    }
+  }
+  acc = warp_sum_u64(acc);
+  if (lane == 0 && acc) atomicAdd(out, (unsigned long long)acc);
+}
+
 // dimension lookup tables (the hash-table build of Crystal's star joins)
 __global__ void k_fill(int32_t* __restrict__ t, uint32_t len, int32_t v) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < len; i += gridDim.x * blockDim.x) t[i] = v;
@@ -1490,6 +1614,33 @@ tp_status tp_plain_sum(const int32_t* d_x, uint64_t n, int64_t* d_sum, void* str
   const int grid = sm_count() * 8;
   k_plain_sum<<<grid, 256, 0, (cudaStream_t)stream>>>(reinterpret_cast<const int4*>(d_x), d_x, n,
                                                       reinterpret_cast<unsigned long long*>(d_sum));
+  return launched();
+}
+
+tp_status tp_bitmap_sum(const tp_column* dcol, const uint32_t* d_bitmap, int64_t* d_sum, void* stream) {
+  if (!dcol || !d_bitmap || !d_sum) return TP_EINVAL;
+  if (dcol->n == 0) return TP_OK;
+  Params P;
+  size_t smem_unused = 0;
+  tp_status st = build_params(dcol, 1, 0, 0, P, smem_unused);
+  if (st != TP_OK) return st;
+  auto out = reinterpret_cast<unsigned long long*>(d_sum);
+  const bool rf = dcol->scheme == TP_RFOR;
+  const size_t smem = rf ? 8u * RFOR_SCRATCH_WORDS * 4u : 0u;
+  const uint32_t npairs = (P.ntiles + 1) / 2;
+  auto go = [&](auto kernel) {
+    cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, 256, smem);
+    const int grid = std::max(1, std::min<int>(sm_count() * std::max(1, occ), (int)((npairs + 7) / 8)));
+    kernel<<<grid, 256, smem, (cudaStream_t)stream>>>(P, d_bitmap, out);
+  };
+  switch (scheme_mask(P)) {
+    case M_FOR: go(k_bitmap_sum<M_FOR>); break;
+    case M_DFOR: go(k_bitmap_sum<M_DFOR>); break;
+    case M_NONE: go(k_bitmap_sum<M_NONE>); break;
+    default: go(k_bitmap_sum<M_RFOR>); break;
+  }
   return launched();
 }
 

@@ -79,6 +79,7 @@ def _load():
         "tp_decode_sum": (i32, [colp, vp, vp]),
         "tp_select_project_sum": (i32, [colp, i32, vp, vp, i32, i32, i32, vp, vp]),
         "tp_plain_sum": (i32, [vp, u64, vp, vp]),
+        "tp_bitmap_sum": (i32, [colp, vp, vp, vp]),
         "tp_cascaded_workspace_words": (u64, [colp]),
         "tp_decode_cascaded": (i32, [colp, vp, vp, vp]),
         "tp_lookup_build": (i32, [vp, u64, ctypes.c_int32, u32, ctypes.POINTER(tp_dim_pred), i32, vp, vp, vp]),
@@ -262,6 +263,19 @@ def tp_gpu_encode(scheme: int, d_x, n: int, starts0, data0, cap0: int, starts1, 
     _check(_lib.tp_gpu_encode(scheme, _ptr(d_x), n, _ptr(starts0), _ptr(data0), cap0, _ptr(starts1), _ptr(data1),
                               cap1, _ptr(d_work), ctypes.byref(col), _stream(stream)), "tp_gpu_encode")
     return col
+
+
+def tp_bitmap_sum(dcol: tp_column, d_bitmap, d_sum, stream=None):
+    _check(_lib.tp_bitmap_sum(ctypes.byref(dcol), _ptr(d_bitmap), _ptr(d_sum), _stream(stream)), "tp_bitmap_sum")
+
+
+def bitmap_sum(dcol, d_bitmap, out=None, stream=None):
+    """Random access: sum of the rows selected by a device bitvector."""
+    import torch
+    if out is None:
+        out = torch.zeros(1, dtype=torch.int64, device=dcol.data0.device)
+    tp_bitmap_sum(dcol.col, d_bitmap, out, stream)
+    return out
 
 
 def tp_plain_sum(d_x, n: int, d_sum, stream=None):

@@ -172,3 +172,22 @@ def test_none_plain_column(n):
     got = int(tp.select_project_sum([d, d], [-(2**30), 0], [2**30, 2**31 - 1], "col", 1, 0).item())
     want = oracle.select_project_sum([x, x], [-(2**30), 0], [2**30, 2**31 - 1], "col", 1, 0)
     assert got == want
+
+
+@pytest.mark.parametrize("scheme", ("for", "dfor", "rfor", "none"))
+def test_bitmap_random_access(scheme):
+    """NEXT-4 random access: the sum of the rows a predicate bitvector selects,
+    across selectivities from 0 (every tile skipped) to 1, ragged tail, == the oracle."""
+    for n in (512 * 301 + 77, 2_000_003):
+        x = {"for": datagen.uniform_bits(17, n, seed=1), "dfor": datagen.near_sorted(n, seed=2),
+             "rfor": datagen.runs(n, 9, seed=3), "none": datagen.uniform_bits(31, n, seed=4)}[scheme]
+        d = tp.encode(x, scheme).to_device()
+        for k, sigma in enumerate((0.0, 1e-5, 1 / 512, 0.01, 0.3, 1.0)):
+            bm = datagen.bernoulli_bitmap(n, sigma, seed=10 + k)
+            got = int(tp.bitmap_sum(d, torch.from_numpy(bm.view(np.int32)).cuda()).item())
+            assert got == oracle.bitmap_sum(x, bm), (scheme, n, sigma)
+    # one selected row in the last, partial miniblock; bits past n set (ignored)
+    bm = np.zeros((n + 31) // 32, np.uint32)
+    bm[-1] = np.uint32(0xffffffff)
+    got = int(tp.bitmap_sum(d, torch.from_numpy(bm.view(np.int32)).cuda()).item())
+    assert got == int(x[(n // 32) * 32:].astype(np.int64).sum())

@@ -211,3 +211,26 @@ def test_choose_scheme_gpu_star():
     assert oracle.choose_scheme(datagen.d1_prefix(100_000, 2**28, 250_000_000))[0] == "dfor"
     assert oracle.choose_scheme(datagen.runs(100_000, 32, seed=1))[0] == "rfor"
     assert oracle.choose_scheme(datagen.uniform_bits(12, 100_000, seed=1))[0] == "for"
+
+
+def test_bitmap_sum_pins():
+    """Random-access oracle: all-ones == the column sum, all-zeros == 0, a
+    bitvector built from a predicate == the SQL select/sum of the same predicate (pins the
+    LSB-first bit order against the independent select oracle), single bits == single rows."""
+    x = datagen.uniform_bits(20, 10_000 + 17, seed=3)
+    n = len(x)
+    ones = datagen.bernoulli_bitmap(n, 1.0)
+    assert oracle.bitmap_sum(x, ones) == oracle.column_sum(x)
+    assert oracle.bitmap_sum(x, datagen.bernoulli_bitmap(n, 0.0)) == 0
+    pred = (x >= 1000) & (x <= 300_000)
+    words = np.zeros((n + 31) // 32, np.uint32)
+    for i in np.flatnonzero(pred):
+        words[i // 32] |= np.uint32(1 << (i % 32))
+    assert oracle.bitmap_sum(x, words) == oracle.select_project_sum([x], [1000], [300_000], "col", 0)
+    for i in (0, 31, 32, n - 1):
+        w = np.zeros((n + 31) // 32, np.uint32)
+        w[i // 32] = np.uint32(1 << (i % 32))
+        assert oracle.bitmap_sum(x, w) == int(x[i])
+    bm = datagen.bernoulli_bitmap(n, 0.01, seed=4)
+    frac = np.unpackbits(bm.view(np.uint8), bitorder="little")[:n].mean()
+    assert 0.005 < frac < 0.02
