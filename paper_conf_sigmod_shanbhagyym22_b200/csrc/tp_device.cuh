@@ -216,8 +216,28 @@ __device__ __forceinline__ void unpack_any(const uint32_t* __restrict__ w, uint3
 // Warp-cooperative dispatch: the warp runs the specialised routine once per
 // distinct bitwidth among its lanes (one pass when the column's miniblocks share b,
 // the common case; a few passes for sorted-delta or run-length streams).
+#ifndef TP_UNPACK_MAX_PASSES
+#define TP_UNPACK_MAX_PASSES 2
+#endif
 __device__ __forceinline__ void unpack_mb(const uint32_t* __restrict__ w, uint32_t b, uint32_t (&e)[32]) {
   uint32_t todo = FULL;
+#if TP_UNPACK_MAX_PASSES < 32
+  // more distinct bitwidths than TP_UNPACK_MAX_PASSES among the lanes (delta streams of
+  // near-sorted keys): one runtime-bitwidth pass beats several specialised ones
+  {
+    uint32_t t = FULL;
+#pragma unroll
+    for (int k = 0; k < TP_UNPACK_MAX_PASSES; ++k) {
+      const uint32_t bl = __shfl_sync(FULL, b, __ffs(t) - 1);
+      t &= ~__ballot_sync(FULL, b == bl);
+      if (t == 0u) break;  // (warp-uniform)
+    }
+    if (t) {
+      unpack_any(w, b, e);
+      return;
+    }
+  }
+#endif
   do {
     const uint32_t bl = __shfl_sync(FULL, b, __ffs(todo) - 1);
     const bool mine = b == bl;
