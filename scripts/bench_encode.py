@@ -23,6 +23,9 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 import datagen  # noqa: E402
+import oracle  # noqa: E402  (cpu_baseline: the oracle's encoder timed beside the GPU, bounded sample)
+
+ORACLE_SAMPLE = 20_000_000  # rows of each column the oracle encodes (1 thread, ~1-3 s)
 
 
 def configs(rows):
@@ -108,6 +111,13 @@ def main():
              "gpu_encode_hbm_gbs": alg / ms / 1e6, "gpu_encode_hbm_frac": alg / ms / 1e6 / peak,
              "gpu_sizes_all3_ms": ms_sizes, "gpu_sizes_hbm_frac": 4 * n / ms_sizes / 1e6 / peak,
              "host_encode_s": host_s, "gpu_vs_host": host_s * 1e3 / ms, "parity": ok}
+        import time as _t
+        t1 = _t.perf_counter()
+        oracle.encode(scheme, x[:ORACLE_SAMPLE])
+        osec = _t.perf_counter() - t1
+        r["oracle_encode_rows_per_s"] = min(n, ORACLE_SAMPLE) / osec
+        r["oracle_sample_rows"] = min(n, ORACLE_SAMPLE)
+        r["gpu_vs_oracle"] = (n / (ms / 1e3)) / r["oracle_encode_rows_per_s"]
         res["configs"][name] = r
         print(name, json.dumps({k: (round(v, 4) if isinstance(v, float) else v) for k, v in r.items()}), flush=True)
         del xd, s0, d0, s1, d1, h, x

@@ -61,9 +61,14 @@ def main():
                 torch.cuda.synchronize()
                 ts.append(a.elapsed_time(b))
             ms = statistics.median(ts)
-            ok = int(acc.item()) == oracle.bitmap_sum(x, bm)
+            import time as _t
+            t1 = _t.perf_counter()
+            want = oracle.bitmap_sum(x, bm)  # the oracle's plain definition, timed beside (numpy, host)
+            osec = _t.perf_counter() - t1
+            ok = int(acc.item()) == want
             p = {"sigma": sigma, "column": name, "ms": ms, "compressed_bytes": d.nbytes(),
-                 "full_scan_frac": (d.nbytes() + n / 8) / ms / 1e6 / peak, "parity": ok}
+                 "full_scan_frac": (d.nbytes() + n / 8) / ms / 1e6 / peak, "parity": ok,
+                 "oracle_ms": osec * 1e3}
             res["points"].append(p)
             print(json.dumps({k: (round(v, 5) if isinstance(v, float) else v) for k, v in p.items()}), flush=True)
     if args.out:
