@@ -42,13 +42,16 @@ constexpr int ETHREADS = 32 * EW;
 constexpr uint64_t ST_AGG = 1ull << 62, ST_INC = 2ull << 62, ST_VAL = (1ull << 62) - 1;
 constexpr int MODE_SIZES = 0;                          // SCHEME template value: all three plans, counts only
 
-// tiles per warp: FOR / DFOR -- 2 (lane l owns miniblock l & 15 of tile l >> 4, the decoder's
-// mapping); RFOR and the sizes pass -- 1 (the run scan takes the whole warp; for packing, lanes
-// 0-15 own the value stream's miniblocks and lanes 16-31 the run-length stream's)
-__host__ __device__ constexpr int tpw_of(int scheme) { return scheme == TP_FOR || scheme == TP_DFOR ? 2 : 1; }
+// tiles per warp: 2 (lane l owns miniblock l & 15 of tile l >> 4, the decoder's mapping)
+__host__ __device__ constexpr int tpw_of(int) { return 2; }
+constexpr uint32_t STG_TILE = 528;
+// RFOR / sizes: three regions per warp -- X (the 2 staged tiles, then the value stream's
+// output staging), V (run values of both tiles, then the run-length stream's staging), L
+// (run lengths); a tile's stream output <= 6 + 512 words, staged at tile * RF_STG
+constexpr uint32_t RF_REGION = 1040, RF_STG = 520;
 // sub-rounds per chunk: FOR / DFOR warps stage and pack 2 x 2 tiles before the chunk's
 // look-back (halves the look-back waits per row, measured); RFOR packs from registers after it
-__host__ __device__ constexpr int ks_of(int scheme) { return tpw_of(scheme) == 2 ? 2 : 1; }
+__host__ __device__ constexpr int ks_of(int scheme) { return scheme == TP_FOR || scheme == TP_DFOR ? 2 : 1; }
 __host__ __device__ constexpr uint32_t chunk_rows(int scheme) {
   return EW * tpw_of(scheme) * ks_of(scheme) * TILE_ROWS;
 }
@@ -56,9 +59,8 @@ __host__ __device__ constexpr uint32_t chunk_rows(int scheme) {
 // the output staging (2 x 528 >= 2 x (1 + 4 (2 + 128)) words) + 16 relative block starts;
 // RFOR / sizes: X, run starts S, V, L
 __host__ __device__ constexpr uint32_t warp_words(int scheme) {
-  return tpw_of(scheme) == 2 ? 1056u * ks_of(scheme) + 16u : 2048u;
+  return scheme == TP_FOR || scheme == TP_DFOR ? 1056u * ks_of(scheme) + 16u : 3u * RF_REGION;
 }
-constexpr uint32_t STG_TILE = 528;
 
 // workspace (u64 words): [0] chunk counter, [1..2] stream totals, [3..4] max tile words,
 // [5] overflow flag, [6..9] sizes mode: FOR, DFOR, RFOR values, RFOR lengths; then the
@@ -169,30 +171,43 @@ __device__ __forceinline__ void plan_for_mb(const uint32_t (&v)[32], uint32_t j,
   b = bitlen(o);
 }
 
-// runs of one 512-row tile (R18; X staged with xs): V[xs(e)] = value of run e, L[xs(e)] =
-// its length; returns r.  S = scratch (run start rows).
-__device__ uint32_t find_runs(const uint32_t* X, uint32_t m, uint32_t* V, uint32_t* S, uint32_t* L,
-                              uint32_t lane) {
-  uint32_t base = 0u;
-  const uint32_t lt = (1u << lane) - 1u;
-#pragma unroll 1
-  for (uint32_t q = 0; q < 16; ++q) {
-    if (32u * q >= m) break;  // warp-uniform
-    const uint32_t row = 32u * q + lane;
-    const uint32_t xv = X[xs(row)];
-    const bool f = row < m && (row == 0 || xv != X[xs(row - 1)]);
-    const uint32_t bal = __ballot_sync(FULL, f);
-    if (f) {
-      const uint32_t e = base + __popc(bal & lt);
-      V[xs(e)] = xv;
-      S[e] = row;
-    }
-    base += __popc(bal);
+// runs of the lane's tile (R18), lane j = miniblock j (rows 32 j .. 32 j + 31 of the tile,
+// values v): the lane marks the rows of its miniblock that start a run (32-bit mask), a
+// 16-lane scan of the mark counts numbers the runs, and the lane writes its runs' values
+// (read back from the staged rows X, xs layout, tile base row xrow0) and lengths (up to the
+// next start -- in its mask, else the first start of a later miniblock, a 16-lane suffix
+// min) to Vt[xs(e)], Lt[xs(e)].  Returns r (uniform over the 16 lanes).
+__device__ __forceinline__ uint32_t runs_mb(const uint32_t (&v)[32], const uint32_t* X, uint32_t xrow0, uint32_t j,
+                                            uint32_t m, uint32_t* Vt, uint32_t* Lt, uint32_t lane) {
+  const uint32_t row0 = 32u * j;
+  const uint32_t prev = __shfl_up_sync(FULL, v[31], 1);  // the previous miniblock's last row
+  uint32_t mask = 0u;
+#pragma unroll
+  for (int i = 0; i < 32; ++i) {
+    const uint32_t pv = i ? v[i - 1] : prev;
+    const bool f = row0 + i < m && ((i == 0 && j == 0) || v[i] != pv);
+    mask |= (uint32_t)f << i;
   }
-  __syncwarp();
-  for (uint32_t e = lane; e < base; e += 32) L[xs(e)] = (e + 1 < base ? S[e + 1] : m) - S[e];
-  __syncwarp();
-  return base;
+  uint32_t r;
+  uint32_t e = excl16(__popc(mask), lane, &r);
+  uint32_t s = mask ? row0 + __ffs(mask) - 1u : m;  // first start at or after this miniblock
+#pragma unroll
+  for (int d = 1; d < 16; d <<= 1) {
+    const uint32_t y = __shfl_down_sync(FULL, s, d);
+    if ((lane & 15u) + d < 16u) s = min(s, y);
+  }
+  uint32_t nf = __shfl_down_sync(FULL, s, 1);  // first start after this miniblock
+  if ((lane & 15u) == 15u) nf = m;
+  uint32_t mm = mask;
+  while (mm) {
+    const uint32_t i = __ffs(mm) - 1u;
+    mm &= mm - 1u;
+    const uint32_t end = mm ? row0 + __ffs(mm) - 1u : nf;
+    Vt[xs(e)] = X[xs(xrow0 + row0 + i)];
+    Lt[xs(e)] = end - (row0 + i);
+    ++e;
+  }
+  return r;
 }
 
 // RFOR plan of the lane's miniblock j (16 tight miniblocks of 32 entries, R17) of the stream
@@ -274,11 +289,12 @@ template <int SCHEME>
 __global__ void __launch_bounds__(ETHREADS, 3) k_encode(const __grid_constant__ EncArgs<SCHEME> A) {
   extern __shared__ __align__(16) uint32_t esm[];
   constexpr bool SIZES = SCHEME == MODE_SIZES;
-  constexpr int TPW = tpw_of(SCHEME);   // tiles per warp and sub-round
+  constexpr bool RF = SCHEME == TP_RFOR;
+  constexpr int TPW = tpw_of(SCHEME);   // tiles per warp and sub-round (2)
   constexpr int KS = ks_of(SCHEME);     // sub-rounds per chunk (staged side by side)
   constexpr int TW = TPW * KS;          // tiles per warp and chunk
   constexpr bool DF = SCHEME == TP_DFOR;
-  constexpr int NS = SCHEME == TP_RFOR ? 2 : 1;
+  constexpr int NS = RF ? 2 : 1;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
   const uint32_t seg = lane >> 4, j = lane & 15u;
   __shared__ uint32_t s_chunk;
@@ -297,17 +313,14 @@ __global__ void __launch_bounds__(ETHREADS, 3) k_encode(const __grid_constant__ 
     uint32_t u[32];
     uint32_t b = 0u, P = 0u, nw = 0u;  // bitwidth, data-word offset, words of the lane's miniblock
     int32_t ref = 0;
-    uint32_t wv = 0u, wl = 0u, r = 0u, my_t = t0;
+    uint32_t my_t = t0, r = 0u;
 #pragma unroll 1
     for (uint32_t p = 0; p < (uint32_t)KS; ++p) {
-      uint32_t* X = Xw + p * 1056u;
-      uint32_t* S = X + 512;  // RFOR / sizes: run starts, then V, L
-      uint32_t* V = X + 1024;
-      uint32_t* L = X + 1536;
+      uint32_t* X = Xw + p * (RF || SIZES ? 0u : 1056u);
       const uint32_t tp0 = t0 + p * TPW;
       const uint32_t r0 = tp0 * TILE_ROWS;
       const uint32_t mrows = tp0 < A.ntiles ? min((uint32_t)(TPW * TILE_ROWS), A.n - r0) : 0u;
-      // ---- stage the tiles (coalesced 16-byte loads, miniblock-major swizzled rows)
+      // ---- stage the 2 tiles (coalesced 16-byte loads, miniblock-major swizzled rows)
       if (mrows == TPW * TILE_ROWS) {
         const int4* src = reinterpret_cast<const int4*>(A.x + r0);
         int4 q[4 * TPW];
@@ -320,74 +333,101 @@ __global__ void __launch_bounds__(ETHREADS, 3) k_encode(const __grid_constant__ 
           X[xs(rr)] = rr < mrows ? (uint32_t)A.x[r0 + rr] : 0u;
       }
       __syncwarp();
-      // the lane's tile (FOR / DFOR: tile tp0 + seg; else tp0)
-      my_t = tp0 + (TPW == 2 ? seg : 0u);
+      // the lane's tile and miniblock
+      my_t = tp0 + seg;
       const uint32_t m = my_t < A.ntiles ? min((uint32_t)TILE_ROWS, A.n - my_t * TILE_ROWS) : 0u;
       const uint32_t nblk = (m + 127u) >> 7;
-      uint32_t tw = 0u, first = 0u, wf = 0u, wd = 0u;
-      if (SIZES || SCHEME == TP_FOR || SCHEME == TP_DFOR) {
-        uint32_t v[32];
-        load_mb(X, (TPW == 2 ? 16u * seg : 0u) + j, v);
-        first = v[0];
-        if (SIZES || SCHEME == TP_FOR) {
-          plan_for_mb(v, j, m, u, b, ref);
-          const uint32_t bj = (j >> 2) < nblk ? b : 0u;
-          uint32_t tot;
-          P = excl16(bj, lane, &tot);
-          nw = bj;
-          tw = 2u * nblk + tot;
-          wf = tw;
-        }
-        if (SIZES || SCHEME == TP_DFOR) {
-          // delta slots (R12, R13): slot s = x[s+1] - x[s] for s < m - 1, neutral pads after
-          const uint32_t nxt = __shfl_down_sync(FULL, v[0], 1);
-#pragma unroll
-          for (int i = 0; i < 31; ++i) v[i] = v[i + 1] - v[i];
-          v[31] = nxt - v[31];
-          plan_for_mb(v, j, m ? m - 1u : 0u, u, b, ref);
-          const uint32_t bj = (j >> 2) < nblk ? b : 0u;
-          uint32_t tot;
-          P = excl16(bj, lane, &tot);
-          nw = bj;
-          tw = m > 0 ? 1u + 2u * nblk + tot : 0u;  // first value + blocks (no tile: no words)
-          wd = tw;
-        }
-        if (!SIZES) {
-          __syncwarp();  // every lane holds its rows: the staged tiles become the output staging
-          uint32_t* stg = X + seg * STG_TILE;
-          const uint32_t blk = j >> 2, d0 = DF ? 1u : 0u;
-          const uint32_t bw = bw_word(b, lane);  // (warp-collective: outside the per-tile branch)
-          if (m > 0) {
-            if (DF && j == 0) stg[0] = first;  // first value of the tile
-            if ((j & 3u) == 0 && blk < nblk) {
-              const uint32_t bs = d0 + 2u * blk + P;  // header of block blk (P = its first mb's offset)
-              stg[bs] = (uint32_t)ref;
-              stg[bs + 1] = bw;
-              bsr[4u * (p * TPW + seg) + blk] = bs;
-            }
-          }
-          // one call site for every lane (warp-collective dispatch); nw = 0 past the column's end
-          pack_mb(u, nw, stg + d0 + 2u * (blk + 1u) + P, nw);
-          if (j == 0) s_words[0][TW * warp + p * TPW + seg] = tw;
-        }
-      }
-      if (SIZES || SCHEME == TP_RFOR) {
-        uint32_t cnt = 0u;
-        if (m > 0) r = find_runs(X, m, V, S, L, lane);
-        plan_rfor_mb(seg ? L : V, j, r, u, b, ref, cnt);
-        nw = (cnt * b + 31u) >> 5;  // tight: ceil(cnt b / 32) words
+      uint32_t v[32];
+      load_mb(X, 16u * seg + j, v);
+      uint32_t tw = 0u, wf = 0u, wd = 0u;
+      if (SIZES || SCHEME == TP_FOR) {
+        plan_for_mb(v, j, m, u, b, ref);
+        const uint32_t bj = (j >> 2) < nblk ? b : 0u;
         uint32_t tot;
-        P = excl16(nw, lane, &tot);
-        tw = m > 0 ? 6u + tot : 0u;
-        wv = __shfl_sync(FULL, tw, 0);
-        wl = __shfl_sync(FULL, tw, 16);
-        if (!SIZES && lane == 0) { s_words[0][warp] = wv; s_words[1][warp] = wl; }
+        P = excl16(bj, lane, &tot);
+        nw = bj;
+        tw = 2u * nblk + tot;
+        wf = tw;
       }
-      if (SIZES && lane == 0 && m > 0) {
-        atomicAdd(work + W_SIZES + 0, (unsigned long long)wf);
-        atomicAdd(work + W_SIZES + 1, (unsigned long long)wd);
-        atomicAdd(work + W_SIZES + 2, (unsigned long long)wv);
-        atomicAdd(work + W_SIZES + 3, (unsigned long long)wl);
+      if (SIZES || RF) {
+        // runs of the tile (before the DFOR plan below rewrites v)
+        uint32_t* V = Xw + RF_REGION;
+        uint32_t* L = Xw + 2u * RF_REGION;
+        r = runs_mb(v, X, 512u * seg, j, m, V + 512u * seg, L + 512u * seg, lane);
+      }
+      if (SIZES || DF) {
+        const uint32_t first = v[0];
+        // delta slots (R12, R13): slot s = x[s+1] - x[s] for s < m - 1, neutral pads after
+        const uint32_t nxt = __shfl_down_sync(FULL, v[0], 1);
+#pragma unroll
+        for (int i = 0; i < 31; ++i) v[i] = v[i + 1] - v[i];
+        v[31] = nxt - v[31];
+        plan_for_mb(v, j, m ? m - 1u : 0u, u, b, ref);
+        const uint32_t bj = (j >> 2) < nblk ? b : 0u;
+        uint32_t tot;
+        P = excl16(bj, lane, &tot);
+        nw = bj;
+        tw = m > 0 ? 1u + 2u * nblk + tot : 0u;  // first value + blocks (no tile: no words)
+        wd = tw;
+        if (DF) v[0] = first;
+      }
+      if (SCHEME == TP_FOR || DF) {
+        __syncwarp();  // every lane holds its rows: the staged tiles become the output staging
+        uint32_t* stg = X + seg * STG_TILE;
+        const uint32_t blk = j >> 2, d0 = DF ? 1u : 0u;
+        const uint32_t bw = bw_word(b, lane);  // (warp-collective: outside the per-tile branch)
+        if (m > 0) {
+          if (DF && j == 0) stg[0] = v[0];  // first value of the tile
+          if ((j & 3u) == 0 && blk < nblk) {
+            const uint32_t bs = d0 + 2u * blk + P;  // header of block blk (P = its first mb's offset)
+            stg[bs] = (uint32_t)ref;
+            stg[bs + 1] = bw;
+            bsr[4u * (p * TPW + seg) + blk] = bs;
+          }
+        }
+        // one call site for every lane (warp-collective dispatch); nw = 0 past the column's end
+        pack_mb(u, nw, stg + d0 + 2u * (blk + 1u) + P, nw);
+        if (j == 0) s_words[0][TW * warp + p * TPW + seg] = tw;
+      }
+      if (SIZES || RF) {
+        // the two streams (R17): plan (and, encoding, pack into the staging) the value stream,
+        // then the run-length stream; stream s of tile seg staged at region s, seg * RF_STG
+        __syncwarp();
+        uint32_t wst[2];
+#pragma unroll 1
+        for (uint32_t sidx = 0; sidx < 2; ++sidx) {
+          const uint32_t* E = Xw + (1u + sidx) * RF_REGION + 512u * seg;
+          uint32_t cnt;
+          plan_rfor_mb(E, j, r, u, b, ref, cnt);
+          nw = (cnt * b + 31u) >> 5;  // tight: ceil(cnt b / 32) words
+          uint32_t tot;
+          P = excl16(nw, lane, &tot);
+          wst[sidx] = m > 0 ? 6u + tot : 0u;
+          if (RF) {
+            __syncwarp();  // the region being staged into is read no more
+            uint32_t* stg = Xw + sidx * RF_REGION + seg * RF_STG;
+            const uint32_t bw = bw_word(b, lane);
+            if (m > 0) {
+              if (j == 0) { stg[0] = r; stg[1] = (uint32_t)ref; }
+              if ((j & 3u) == 0) stg[2 + (j >> 2)] = bw;
+            }
+            pack_mb(u, m > 0 ? b : 0u, stg + 6 + P, m > 0 ? nw : 0u);
+            if (j == 0) s_words[sidx][TPW * warp + seg] = wst[sidx];
+          }
+        }
+        if (SIZES) {
+          // one atomic per warp and scheme stream: both tiles' words
+          const uint32_t fv = __shfl_sync(FULL, wf, 0) + __shfl_sync(FULL, wf, 16);
+          const uint32_t dv = __shfl_sync(FULL, wd, 0) + __shfl_sync(FULL, wd, 16);
+          const uint32_t vv = __shfl_sync(FULL, wst[0], 0) + __shfl_sync(FULL, wst[0], 16);
+          const uint32_t lv = __shfl_sync(FULL, wst[1], 0) + __shfl_sync(FULL, wst[1], 16);
+          if (lane == 0 && mrows > 0) {
+            atomicAdd(work + W_SIZES + 0, (unsigned long long)fv);
+            atomicAdd(work + W_SIZES + 1, (unsigned long long)dv);
+            atomicAdd(work + W_SIZES + 2, (unsigned long long)vv);
+            atomicAdd(work + W_SIZES + 3, (unsigned long long)lv);
+          }
+        }
       }
     }
     if (SIZES) {
@@ -416,68 +456,57 @@ __global__ void __launch_bounds__(ETHREADS, 3) k_encode(const __grid_constant__ 
         if (c == A.nchunks - 1) work[W_TOT + warp] = base + agg;
       }
     }
-    if (SCHEME != TP_RFOR && threadIdx.x == 0) s_base[1] = s_agg[1] = 0;
+    if (!RF && threadIdx.x == 0) s_base[1] = s_agg[1] = 0;
     __syncthreads();
-    const bool ovf = s_base[0] + s_agg[0] > A.cap0 || (SCHEME == TP_RFOR && s_base[1] + s_agg[1] > A.cap1);
+    const bool ovf = s_base[0] + s_agg[0] > A.cap0 || (RF && s_base[1] + s_agg[1] > A.cap1);
     if (t0 < A.ntiles && !ovf) {
-      // the warp's base word in each stream: the chunk base + the earlier tiles of the chunk
-      uint64_t B0 = s_base[0], B1 = s_base[1];
-      for (uint32_t k = 0; k < TW * warp; ++k) B0 += s_words[0][k];
-      for (uint32_t k = 0; k < warp && SCHEME == TP_RFOR; ++k) B1 += s_words[1][k];
-      uint64_t e0 = B0, e1 = B1 + wl;  // end of the warp's words
-      if (SCHEME == TP_RFOR) {
-        // header [r][ref][4 bitwidth words] and the tight miniblocks, straight from registers
-        const uint64_t Bs = seg ? B1 : B0;
-        uint32_t* data = seg ? A.data1 : A.data0;
-        uint32_t* starts = seg ? A.starts1 : A.starts0;
-        const uint32_t bw = bw_word(b, lane);
-        if (j == 0) {
-          starts[my_t] = (uint32_t)Bs;
-          data[Bs] = r;
-          data[Bs + 1] = (uint32_t)ref;
-        }
-        if ((j & 3u) == 0) data[Bs + 2 + (j >> 2)] = bw;
-        pack_mb(u, b, data + Bs + 6 + P, nw);
-        e0 = B0 + wv;
-      } else {
-        // block_starts (lane 4 tl + blk: block blk of the warp's tile tl), then the staged
-        // words of the warp's tiles, coalesced
-        uint64_t off = 0;
-        const uint32_t tl = lane >> 2, blk = lane & 3u;
-        uint64_t my_off = 0;
+      uint64_t e[2];
+#pragma unroll 1
+      for (uint32_t sidx = 0; sidx < (uint32_t)NS; ++sidx) {
+        uint32_t* data = sidx ? A.data1 : A.data0;
+        uint32_t* starts = sidx ? A.starts1 : A.starts0;
+        // the warp's base word: the chunk base + the earlier tiles of the chunk
+        uint64_t B = s_base[sidx];
+        for (uint32_t k = 0; k < TW * warp; ++k) B += s_words[sidx][k];
+        // block_starts (lane 4 tl + blk: block blk of the warp's tile tl; RFOR: lane tl), then
+        // the staged words of the warp's tiles, coalesced
+        uint64_t off = 0, my_off = 0;
+        const uint32_t tl = RF ? lane : lane >> 2, blk = RF ? 0u : lane & 3u;
 #pragma unroll 1
         for (uint32_t k = 0; k < (uint32_t)TW; ++k) {
           if (k == tl) my_off = off;
-          off += s_words[0][TW * warp + k];
+          off += s_words[sidx][TW * warp + k];
         }
         const uint32_t t = t0 + tl;
         if (tl < (uint32_t)TW && t < A.ntiles) {
-          const uint32_t mt = min((uint32_t)TILE_ROWS, A.n - t * TILE_ROWS);
-          if (blk < ((mt + 127u) >> 7)) A.starts0[4ull * t + blk] = (uint32_t)(B0 + my_off + bsr[lane]);
+          if (RF) {
+            starts[t] = (uint32_t)(B + my_off);
+          } else {
+            const uint32_t mt = min((uint32_t)TILE_ROWS, A.n - t * TILE_ROWS);
+            if (blk < ((mt + 127u) >> 7)) starts[4ull * t + blk] = (uint32_t)(B + my_off + bsr[lane]);
+          }
         }
-        uint64_t o = B0;
+        uint64_t o = B;
 #pragma unroll 1
         for (uint32_t k = 0; k < (uint32_t)TW; ++k) {
-          const uint32_t wk = s_words[0][TW * warp + k];
-          const uint32_t* src = Xw + (k / TPW) * 1056u + (k % TPW) * STG_TILE;
-          for (uint32_t i = lane; i < wk; i += 32) A.data0[o + i] = src[i];
+          const uint32_t wk = s_words[sidx][TW * warp + k];
+          const uint32_t* src = RF ? Xw + sidx * RF_REGION + k * RF_STG : Xw + (k / TPW) * 1056u + (k % TPW) * STG_TILE;
+          for (uint32_t i = lane; i < wk; i += 32) data[o + i] = src[i];
           o += wk;
         }
-        e0 = o;
+        e[sidx] = o;
       }
       // the column's end: last block_starts entry + zero guards (R6, R9)
       if (t0 + TW >= A.ntiles) {
-        if (lane < TP_GUARD_WORDS) {
-          A.data0[e0 + lane] = 0u;
-          A.starts0[A.nblocks + 1 + lane] = 0u;
-          if (SCHEME == TP_RFOR) {
-            A.data1[e1 + lane] = 0u;
-            A.starts1[A.nblocks + 1 + lane] = 0u;
+#pragma unroll 1
+        for (uint32_t sidx = 0; sidx < (uint32_t)NS; ++sidx) {
+          uint32_t* data = sidx ? A.data1 : A.data0;
+          uint32_t* starts = sidx ? A.starts1 : A.starts0;
+          if (lane < TP_GUARD_WORDS) {
+            data[e[sidx] + lane] = 0u;
+            starts[A.nblocks + 1 + lane] = 0u;
           }
-        }
-        if (lane == 0) {
-          A.starts0[A.nblocks] = (uint32_t)e0;
-          if (SCHEME == TP_RFOR) A.starts1[A.nblocks] = (uint32_t)e1;
+          if (lane == 0) starts[A.nblocks] = (uint32_t)e[sidx];
         }
       }
     }
