@@ -51,7 +51,10 @@ constexpr uint32_t STG_TILE = 528;
 constexpr uint32_t RF_REGION = 1040, RF_STG = 520;
 // sub-rounds per chunk: FOR / DFOR warps stage and pack 2 x 2 tiles before the chunk's
 // look-back (halves the look-back waits per row, measured); RFOR packs from registers after it
-__host__ __device__ constexpr int ks_of(int scheme) { return scheme == TP_FOR || scheme == TP_DFOR ? 2 : 1; }
+#ifndef TP_ENC_KS
+#define TP_ENC_KS 2
+#endif
+__host__ __device__ constexpr int ks_of(int scheme) { return scheme == TP_FOR || scheme == TP_DFOR ? TP_ENC_KS : 1; }
 __host__ __device__ constexpr uint32_t chunk_rows(int scheme) {
   return EW * tpw_of(scheme) * ks_of(scheme) * TILE_ROWS;
 }
@@ -298,7 +301,7 @@ __global__ void __launch_bounds__(ETHREADS, 3) k_encode(const __grid_constant__ 
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
   const uint32_t seg = lane >> 4, j = lane & 15u;
   __shared__ uint32_t s_chunk;
-  __shared__ uint32_t s_words[2][EW * 4];
+  __shared__ uint32_t s_words[2][EW * 2 * TP_ENC_KS];
   __shared__ unsigned long long s_base[2], s_agg[2];
   uint32_t* Xw = esm + warp * warp_words(SCHEME);
   uint32_t* bsr = Xw + KS * 1056u;  // FOR / DFOR: block starts relative to their tile, 4 per tile
@@ -438,9 +441,12 @@ __global__ void __launch_bounds__(ETHREADS, 3) k_encode(const __grid_constant__ 
     __syncthreads();
     constexpr int NT = EW * TW;
     if (warp < NS) {
-      const uint32_t mine = lane < NT ? s_words[warp][lane] : 0u;
-      uint64_t agg = mine;
-      uint32_t mx = mine;
+      uint64_t agg = 0;
+      uint32_t mx = 0u;
+      for (uint32_t k = lane; k < (uint32_t)NT; k += 32) {
+        agg += s_words[warp][k];
+        mx = max(mx, s_words[warp][k]);
+      }
 #pragma unroll
       for (int d = 16; d > 0; d >>= 1) {
         agg += __shfl_xor_sync(FULL, agg, d);
