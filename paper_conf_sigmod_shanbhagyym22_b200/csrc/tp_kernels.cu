@@ -614,8 +614,13 @@ struct GlobalOp : OpBase {
     if (pair_tile >= C.tile_end) return;  // warp-uniform
     uint32_t* buf = scratch + P.staging_off;
     buf = reinterpret_cast<uint32_t*>((reinterpret_cast<uintptr_t>(buf) + 1023) & ~uintptr_t(1023));
-    buf += (rc & 1u) * 1024u;
-    if (g.lane == 0) bulk_wait_read<1>();  // the store issued from this buffer two rounds ago is done reading
+    // RFOR: one buffer (its shared-memory budget -- the expansion scratch -- is what keeps a 3rd
+    // CTA per SM; the expansion of the next round covers the store's read), else two
+    constexpr bool SINGLE = MASK == M_RFOR;
+    if (!SINGLE) buf += (rc & 1u) * 1024u;
+    if (g.lane == 0) {  // the store issued from this buffer earlier is done reading it
+      if (SINGLE) bulk_wait_read<0>(); else bulk_wait_read<1>();
+    }
     __syncwarp();
     const uint32_t l = g.lane;
 #pragma unroll
@@ -1458,8 +1463,8 @@ tp_status decode_global_impl(const tp_column* dcol, int32_t* d_out, bool raw, vo
   if (raw && dcol->scheme == TP_RFOR) return TP_EINVAL;
   Params P;
   size_t smem = 0;
-  // per warp: 2 x 4 KB swizzled staging + 1 KB alignment slop
-  tp_status st = build_params(dcol, 1, 2048u + 256u, 0, P, smem);
+  // per warp: 2 x 4 KB swizzled staging (RFOR: 1) + 1 KB alignment slop
+  tp_status st = build_params(dcol, 1, (dcol->scheme == TP_RFOR ? 1024u : 2048u) + 256u, 0, P, smem);
   if (st != TP_OK) return st;
   CUtensorMap tmap;
   memset(&tmap, 0, sizeof(tmap));
