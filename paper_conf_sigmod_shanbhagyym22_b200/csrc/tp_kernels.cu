@@ -545,23 +545,48 @@ struct OpBase {
   __device__ void end(const Params&, const StageCtx&, const Lane&) {}
 };
 
-// decode -> sum (decode-only microbenchmark)
-template <uint32_t MASK>
+// decode -> sum (decode-only microbenchmark).  LEAN (FOR below ~12 bits, where the
+// kernel is instruction-bound): the stream view once per item and a CTA-uniform full-round
+// test instead of a per-lane row mask + vote (measured -3..-10 % at b <= 12; at b = 16, where
+// HBM binds, the plain variant is 2.7 % faster, so it keeps it)
+template <uint32_t MASK, bool LEAN = false>
 struct SumOp : OpBase {
   static constexpr uint32_t kMask = MASK;
   static constexpr bool kProducerSpin = MASK == M_FOR;
   unsigned long long* out;
   uint64_t acc;
+  uint32_t sv_t0s = 0xffffffffu;  // the item whose stream view is cached (FOR)
+  StreamView sv;
   __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t, uint32_t) {
     const Col& c = P.col[0];
-    const uint32_t alive = valid_rows(P, C, g);
     if (MASK == M_FOR) {
-      const StreamView v = stream_view(P, c.s0, C);
-      uint32_t tl;
-      bool tv;
-      const MbView m = for_mb(P, c, C, g, v, tl, tv);
+      MbView m;
+      uint32_t alive;
+      bool full;
+      if constexpr (LEAN) {
+        // per-item work once per item, not once per round (low bitwidths are instruction-bound)
+        if (C.t0s != sv_t0s) {
+          sv = stream_view(P, c.s0, C);
+          sv_t0s = C.t0s;
+        }
+        uint32_t tl;
+        bool tv;
+        m = for_mb(P, c, C, g, sv, tl, tv);
+        // a round whose TPR tiles are all inside the CTA range needs no row mask (CTA-uniform)
+        const uint32_t tend = C.t0s + C.round_base + TPR;
+        const bool full_round = tend <= C.tile_end && tend * (uint32_t)TILE_ROWS <= P.n;
+        alive = full_round ? 0xffffffffu : valid_rows(P, C, g);
+        full = full_round || __all_sync(FULL, alive == 0xffffffffu);
+      } else {
+        alive = valid_rows(P, C, g);
+        const StreamView v = stream_view(P, c.s0, C);
+        uint32_t tl;
+        bool tv;
+        m = for_mb(P, c, C, g, v, tl, tv);
+        full = __all_sync(FULL, alive == 0xffffffffu);
+      }
       // the branch must be warp-uniform: both sides run warp-collective dispatch code
-      if (__all_sync(FULL, alive == 0xffffffffu)) {
+      if (full) {
         const uint64_t se = sum_mb(m.w, m.b);
         acc += se + (uint64_t)((int64_t)(int32_t)m.ref * 32);
       } else {
@@ -572,6 +597,7 @@ struct SumOp : OpBase {
           if (alive & (1u << i)) acc += (uint64_t)(int64_t)(int32_t)(m.ref + e[i]);
       }
     } else {
+      const uint32_t alive = valid_rows(P, C, g);
       uint32_t val[32];
       decode_col<MASK>(P, 0, C, g, scratch, val);
       if (alive == 0xffffffffu) {  // per-lane branch, no collectives inside
@@ -1023,9 +1049,9 @@ struct StarOp : OpBase {
 #ifndef TP_SUM_MINB
 #define TP_SUM_MINB 4
 #endif
-template <uint32_t MASK>
+template <uint32_t MASK, bool LEAN = false>
 __global__ void __launch_bounds__(THREADS, TP_SUM_MINB) k_decode_sum(const __grid_constant__ Params P, unsigned long long* out) {
-  SumOp<MASK> op;
+  SumOp<MASK, LEAN> op;
   op.out = out;
   op.acc = 0;
   run_pipeline(P, op);
@@ -1444,7 +1470,13 @@ tp_status tp_decode_sum(const tp_column* dcol, int64_t* d_sum, void* stream) {
   auto out = reinterpret_cast<unsigned long long*>(d_sum);
   const int cap = (int)((P.ntiles + 1) / 2);
   switch (scheme_mask(P)) {
-    case M_FOR: launch(k_decode_sum<M_FOR>, smem, cap, stream, P, out); break;
+    case M_FOR:
+      // a tile of < 12-bit miniblocks (4 x (2 + 4 x 12) words): the instruction-bound variant
+      if (dcol->max_tile_words0 != 0 && dcol->max_tile_words0 < 200u)
+        launch(k_decode_sum<M_FOR, true>, smem, cap, stream, P, out);
+      else
+        launch(k_decode_sum<M_FOR>, smem, cap, stream, P, out);
+      break;
     case M_DFOR: launch(k_decode_sum<M_DFOR>, smem, cap, stream, P, out); break;
     case M_NONE: launch(k_decode_sum<M_NONE>, smem, cap, stream, P, out); break;
     default: launch(k_decode_sum<M_RFOR>, smem, cap, stream, P, out); break;
