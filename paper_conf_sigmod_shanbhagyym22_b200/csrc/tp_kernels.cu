@@ -1471,8 +1471,9 @@ tp_status tp_decode_sum(const tp_column* dcol, int64_t* d_sum, void* stream) {
   const int cap = (int)((P.ntiles + 1) / 2);
   switch (scheme_mask(P)) {
     case M_FOR:
-      // a tile of < 12-bit miniblocks (4 x (2 + 4 x 12) words): the instruction-bound variant
-      if (dcol->max_tile_words0 != 0 && dcol->max_tile_words0 < 200u)
+      // tiles of <= 12-bit miniblocks (4 x (2 + 4 x 12) words): the instruction-bound variant
+      // (measured: lean -2.5 % at b = 12, +2.7 % at b = 16)
+      if (dcol->max_tile_words0 != 0 && dcol->max_tile_words0 <= 200u)
         launch(k_decode_sum<M_FOR, true>, smem, cap, stream, P, out);
       else
         launch(k_decode_sum<M_FOR>, smem, cap, stream, P, out);
