@@ -191,3 +191,28 @@ def test_bitmap_random_access(scheme):
     bm[-1] = np.uint32(0xffffffff)
     got = int(tp.bitmap_sum(d, torch.from_numpy(bm.view(np.int32)).cuda()).item())
     assert got == int(x[(n // 32) * 32:].astype(np.int64).sum())
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("scheme,gen", [
+    ("dfor", lambda n: datagen.d1_sorted(n, 2**28)),        # BASELINE config 3
+    ("rfor", lambda n: datagen.runs(n, 4)),                 # BASELINE config 4, shortest runs
+])
+def test_full_size_dfor_rfor(scheme, gen):
+    """configs 3 / 4 at the suite's full size (500M rows), in the launch configuration
+    scripts/bench_suite.py times: the GPU decode of the encoded bytes == the oracle's decode of
+    the same bytes (whole column), and the fused sum == the oracle's int64 sum."""
+    n = 500_000_000
+    x = gen(n)
+    h = tp.encode(x, scheme)
+    a = h.arrays()
+    if scheme == "dfor":
+        e = oracle.Encoded(scheme="dfor", header=a["header"], starts=a["starts0"], data=a["data0"])
+    else:
+        e = oracle.Encoded(scheme="rfor", header=a["header"], startsV=a["starts0"], dataV=a["data0"],
+                           startsL=a["starts1"], dataL=a["data1"])
+    want = oracle.decode(e)
+    d = h.to_device()
+    got = tp.decode(d)
+    assert torch.equal(got, torch.from_numpy(want).cuda())
+    assert int(tp.decode_sum(d).item()) == oracle.column_sum(want)
