@@ -54,11 +54,16 @@ typedef enum {
   TP_FOR = 1,   /* GPU-FOR   header [128, 4, n]                          */
   TP_DFOR = 2,  /* GPU-DFOR header [128, 4, n], tiles of D = 4 blocks   */
   TP_RFOR = 3,  /* GPU-RFOR header [512, 16, n], value + run streams     */
-  TP_NONE = 4   /* "None" (Fig. 11): the plain int32 column, header [512, 1, n];
+  TP_NONE = 4,  /* "None" (Fig. 11): the plain int32 column, header [512, 1, n];
                  * block_starts[k] = 512 k (one 512-row tile per block), data = the
                  * values padded with zeros to a multiple of 32 words (words0 = that
                  * padded count).  The uncompressed baseline the paper compares GPU-*
                  * against, run through the same tile pipeline.  Never chosen by GPU-*. */
+  TP_FORNM = 5  /* GPU-FOR WITHOUT miniblocks (the paper's ablation): header
+                 * [128, 1, n]; block = [ref][bitwidth word: byte 0 = b of the whole 128-value
+                 * block][128 entries x b bits, LSB-first] = 2 + 4 b words.  Host encoder and
+                 * decode / decode_sum only (measurement of the miniblock trade-off); never
+                 * chosen by GPU-*, not accepted by the GPU encoder or the query operators. */
 } tp_scheme;
 
 /*

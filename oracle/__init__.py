@@ -191,7 +191,9 @@ def rfor_decode(enc: Encoded) -> np.ndarray:
     return out
 
 
-ENCODERS = {"for": for_encode, "dfor": dfor_encode, "rfor": rfor_encode}
+ENCODERS = {"for": for_encode, "dfor": dfor_encode, "rfor": rfor_encode,
+            # GPU-FOR without miniblocks: one 128-entry miniblock per block
+            "fornm": lambda x: for_encode(x, 128, 1)}
 DECODERS = {"for": for_decode, "dfor": dfor_decode, "rfor": rfor_decode}
 
 

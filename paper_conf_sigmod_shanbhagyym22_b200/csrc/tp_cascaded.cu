@@ -201,7 +201,7 @@ uint64_t tp_cascaded_workspace_words(const tp_column* c) {
 }
 
 tp_status tp_decode_cascaded(const tp_column* c, int32_t* d_out, uint32_t* d_work, void* stream) {
-  if (!c || !d_out || !d_work) return TP_EINVAL;
+  if (!c || !d_out || !d_work || c->scheme == TP_FORNM || c->scheme == TP_NONE) return TP_EINVAL;
   if (c->n == 0) return TP_OK;
   if (c->n >= (1ull << 32)) return TP_EUNSUPPORTED;
   cudaStream_t s = (cudaStream_t)stream;

@@ -30,7 +30,7 @@ constexpr int THREADS = 32 * (CONSUMER_WARPS + 1);
 constexpr int MAX_STREAMS = 2 * 6;  // up to 6 columns, 2 streams each (RFOR)
 constexpr unsigned FULL = 0xffffffffu;
 
-enum : uint32_t { S_FOR = 1, S_DFOR = 2, S_RFOR = 3, S_NONE = 4 };
+enum : uint32_t { S_FOR = 1, S_DFOR = 2, S_RFOR = 3, S_NONE = 4, S_FORNM = 5 };
 
 // ------------------------------------------------------------------ PTX wrappers
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {

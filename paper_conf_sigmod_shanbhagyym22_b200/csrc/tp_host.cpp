@@ -96,6 +96,27 @@ inline uint32_t* write_for_block(const int32_t* v, uint32_t cnt, const ForBlockP
   return out;
 }
 
+// ---- GPU-FOR without miniblocks: one bitwidth per 128-value block
+inline ForBlockPlan plan_fornm_block(const int32_t* v, uint32_t cnt) {
+  ForBlockPlan p{0, 0, 2};
+  if (cnt == 0) return p;
+  int32_t mn = v[0];
+  for (uint32_t i = 1; i < cnt; ++i) mn = std::min(mn, v[i]);
+  uint32_t mx = 0;
+  for (uint32_t i = 0; i < cnt; ++i) mx = std::max(mx, (uint32_t)v[i] - (uint32_t)mn);
+  p.ref = mn;
+  p.bw = bit_length(mx);  // byte 0 (R2 with one miniblock)
+  p.words = 2 + 4 * p.bw;
+  return p;
+}
+inline uint32_t* write_fornm_block(const int32_t* v, uint32_t cnt, const ForBlockPlan& p, uint32_t* out) {
+  *out++ = (uint32_t)p.ref;
+  *out++ = p.bw;
+  BitWriter w(out);
+  for (uint32_t i = 0; i < kBlock; ++i) w.put(i < cnt ? (uint32_t)v[i] - (uint32_t)p.ref : 0u, p.bw);
+  return w.flush();
+}
+
 // ---- GPU-FOR
 struct ForEnc {
   static uint64_t nblocks(uint64_t n) { return (n + kBlock - 1) / kBlock; }
@@ -179,11 +200,14 @@ Sizes compute_sizes(int scheme, const int32_t* x, uint64_t n) {
   if (scheme == TP_NONE) {  // plain values, 512-row tiles, padded to whole 32-row miniblocks
     s.nb = (n + kTile - 1) / kTile;
     s.w0 = (n + 31) / 32 * 32;
-  } else if (scheme == TP_FOR) {
+  } else if (scheme == TP_FOR || scheme == TP_FORNM) {
     s.nb = (n + kBlock - 1) / kBlock;
     s.u0.resize(s.nb);
+    const bool nm = scheme == TP_FORNM;
     parallel_for(s.nb, [&](uint64_t lo, uint64_t hi) {
-      for (uint64_t i = lo; i < hi; ++i) s.u0[i] = ForEnc::block_words(x, n, i);
+      for (uint64_t i = lo; i < hi; ++i)
+        s.u0[i] = nm ? plan_fornm_block(x + i * kBlock, (uint32_t)std::min<uint64_t>(kBlock, n - i * kBlock)).words
+                     : ForEnc::block_words(x, n, i);
     });
     for (uint32_t w : s.u0) s.w0 += w;
   } else if (scheme == TP_DFOR) {
@@ -230,7 +254,7 @@ extern "C" {
 
 tp_status tp_encode_size(int scheme, const int32_t* x, uint64_t n, uint64_t* num_blocks, uint64_t* words0,
                          uint64_t* words1) {
-  if (scheme < TP_FOR || scheme > TP_NONE || (n && !x)) return TP_EINVAL;
+  if (scheme < TP_FOR || scheme > TP_FORNM || (n && !x)) return TP_EINVAL;
   if (n >= (1ull << 32)) return TP_EUNSUPPORTED;
   Sizes s = compute_sizes(scheme, x, n);
   if (s.w0 >= (1ull << 32) || s.w1 >= (1ull << 32)) return TP_EUNSUPPORTED;
@@ -242,7 +266,7 @@ tp_status tp_encode_size(int scheme, const int32_t* x, uint64_t n, uint64_t* num
 
 tp_status tp_encode(int scheme, const int32_t* x, uint64_t n, uint32_t* starts0, uint32_t* data0, uint32_t* starts1,
                     uint32_t* data1, tp_column* out) {
-  if (scheme < TP_FOR || scheme > TP_NONE || (n && !x) || !starts0 || !data0 || !out) return TP_EINVAL;
+  if (scheme < TP_FOR || scheme > TP_FORNM || (n && !x) || !starts0 || !data0 || !out) return TP_EINVAL;
   if (scheme == TP_RFOR && (!starts1 || !data1)) return TP_EINVAL;
   if (n >= (1ull << 32)) return TP_EUNSUPPORTED;
   Sizes s = compute_sizes(scheme, x, n);
@@ -266,19 +290,21 @@ tp_status tp_encode(int scheme, const int32_t* x, uint64_t n, uint32_t* starts0,
     starts0[s.nb] = (uint32_t)s.w0;
     mtw0 = kTile;
     out->block_size = kTile; out->miniblock_count = 1; out->tile_blocks = 1;
-  } else if (scheme == TP_FOR) {
+  } else if (scheme == TP_FOR || scheme == TP_FORNM) {
+    const bool nm = scheme == TP_FORNM;
     parallel_for(s.nb, [&](uint64_t lo, uint64_t hi) {
       for (uint64_t i = lo; i < hi; ++i) {
         const uint32_t cnt = (uint32_t)std::min<uint64_t>(kBlock, n - i * kBlock);
         const int32_t* v = x + i * kBlock;
         starts0[i] = (uint32_t)off0[i];
-        write_for_block(v, cnt, plan_for_block(v, cnt), data0 + off0[i]);
+        if (nm) write_fornm_block(v, cnt, plan_fornm_block(v, cnt), data0 + off0[i]);
+        else write_for_block(v, cnt, plan_for_block(v, cnt), data0 + off0[i]);
       }
     });
     starts0[s.nb] = (uint32_t)s.w0;
     for (uint64_t t = 0; t * 4 < s.nb; ++t)
       mtw0 = std::max<uint32_t>(mtw0, starts0[std::min<uint64_t>(4 * t + 4, s.nb)] - starts0[4 * t]);
-    out->block_size = kBlock; out->miniblock_count = 4; out->tile_blocks = 4;
+    out->block_size = kBlock; out->miniblock_count = nm ? 1 : 4; out->tile_blocks = 4;
   } else if (scheme == TP_DFOR) {
     const uint64_t nt = (n + kTile - 1) / kTile;
     parallel_for(nt, [&](uint64_t lo, uint64_t hi) {

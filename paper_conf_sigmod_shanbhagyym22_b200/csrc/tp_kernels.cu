@@ -80,6 +80,28 @@ __device__ __forceinline__ MbView for_mb(const Params& P, const Col& c, const St
                   g.mb & 3u);
 }
 
+// the thread's 32 rows of a GPU-FOR block WITHOUT miniblocks: one bitwidth b for
+// the block's 128 entries, so quarter j of the block starts at word 2 + j b (the same stream
+// layout as 4 miniblocks of equal width)
+__device__ __forceinline__ MbView fornm_mb(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
+                                           const StreamView& v, uint32_t& tl, bool& tv) {
+  tl = C.round_base + g.tile_local;
+  tv = C.t0s + tl < C.tile_end;
+  const uint32_t lb = 4u * tl + (g.mb >> 2);
+  MbView m;
+  m.valid = tv && 4u * C.t0s + lb < c.nblocks;
+  if (m.valid) {
+    const uint32_t bs = v.ss[v.sshift + lb];
+    const uint32_t* blk = v.sd + (bs - v.lo + v.dshift);
+    m.ref = blk[0];
+    m.b = min(blk[1] & 255u, 32u);
+    m.w = blk + 2u + (g.mb & 3u) * m.b;
+  } else {
+    m.ref = 0u; m.b = 0u; m.w = v.sd;
+  }
+  return m;
+}
+
 // ---------------------------------------------------------------- GPU-FOR decode
 // LoadBitPack analogue: the thread's 32 rows of the tile.
 // COMPACT: multi-column query kernels unpack with the runtime-bitwidth routine (one small
@@ -88,13 +110,13 @@ __device__ __forceinline__ MbView for_mb(const Params& P, const Col& c, const St
 // stalls in the SSB kernel)
 // RAW: the packed offsets only (no reference added) -- the first pass of the cascading
 // baseline (tp_cascaded.cu), also for the delta blocks of a GPU-DFOR column
-template <bool COMPACT, bool RAW = false>
+template <bool COMPACT, bool RAW = false, bool NOMB = false>
 __device__ __forceinline__ void decode_for(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                            uint32_t (&val)[32]) {
   const StreamView v = stream_view(P, c.s0, C);
   uint32_t tl;
   bool tv;
-  const MbView m = for_mb(P, c, C, g, v, tl, tv);
+  const MbView m = NOMB ? fornm_mb(P, c, C, g, v, tl, tv) : for_mb(P, c, C, g, v, tl, tv);
   uint32_t e[32];
   if (COMPACT) unpack_any(m.w, m.b, e); else unpack_mb(m.w, m.b, e);
 #pragma unroll
@@ -327,6 +349,7 @@ __device__ __forceinline__ uint32_t none_at(const uint32_t* w, uint32_t sw, uint
 // MASK: which decoders a kernel instantiation carries (bit 1 << scheme); kernels
 // are instantiated per scheme mix so that FOR-only kernels keep FOR's register budget.
 constexpr uint32_t M_FOR = 1u << S_FOR, M_DFOR = 1u << S_DFOR, M_RFOR = 1u << S_RFOR, M_NONE = 1u << S_NONE;
+constexpr uint32_t M_FORNM = 1u << S_FORNM;  // decode / decode_sum only (the miniblock ablation)
 constexpr uint32_t M_RAW = 1u << 8;  // FOR / DFOR blocks, packed offsets only (cascading baseline)
 template <uint32_t MASK, bool COMPACT = false>
 __device__ __forceinline__ void decode_col(const Params& P, uint32_t ci, const StageCtx& C, const Lane& g,
@@ -334,6 +357,10 @@ __device__ __forceinline__ void decode_col(const Params& P, uint32_t ci, const S
   const Col& c = P.col[ci];
   if (MASK == M_RAW) {
     decode_for<false, true>(P, c, C, g, val);
+    return;
+  }
+  if (MASK == M_FORNM) {
+    decode_for<false, false, true>(P, c, C, g, val);
     return;
   }
   if ((MASK & M_NONE) && c.scheme == S_NONE) decode_none(P, c, C, g, val);
@@ -552,14 +579,14 @@ struct OpBase {
 template <uint32_t MASK, bool LEAN = false>
 struct SumOp : OpBase {
   static constexpr uint32_t kMask = MASK;
-  static constexpr bool kProducerSpin = MASK == M_FOR;
+  static constexpr bool kProducerSpin = MASK == M_FOR || MASK == M_FORNM;
   unsigned long long* out;
   uint64_t acc;
   uint32_t sv_t0s = 0xffffffffu;  // the item whose stream view is cached (FOR)
   StreamView sv;
   __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t, uint32_t) {
     const Col& c = P.col[0];
-    if (MASK == M_FOR) {
+    if (MASK == M_FOR || MASK == M_FORNM) {
       MbView m;
       uint32_t alive;
       bool full;
@@ -582,7 +609,7 @@ struct SumOp : OpBase {
         const StreamView v = stream_view(P, c.s0, C);
         uint32_t tl;
         bool tv;
-        m = for_mb(P, c, C, g, v, tl, tv);
+        m = MASK == M_FORNM ? fornm_mb(P, c, C, g, v, tl, tv) : for_mb(P, c, C, g, v, tl, tv);
         full = __all_sync(FULL, alive == 0xffffffffu);
       }
       // the branch must be warp-uniform: both sides run warp-collective dispatch code
@@ -1291,7 +1318,7 @@ static PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
 
 static uint32_t worst_tile_words(uint32_t scheme) {
   if (scheme == TP_NONE) return TILE_ROWS;
-  return scheme == TP_FOR ? 4u * (2u + 128u) : scheme == TP_DFOR ? 1u + 4u * (2u + 128u) : 6u + 512u;
+  return scheme == TP_FOR || scheme == TP_FORNM ? 4u * (2u + 128u) : scheme == TP_DFOR ? 1u + 4u * (2u + 128u) : 6u + 512u;
 }
 static uint32_t align4(uint32_t w) { return (w + 3u) & ~3u; }
 
@@ -1318,6 +1345,9 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
       if (reinterpret_cast<uintptr_t>(k.data0) & 15u) return TP_EINVAL;
     } else if (k.scheme == TP_FOR || k.scheme == TP_DFOR) {
       if (k.block_size != 128 || k.miniblock_count != 4 || k.num_blocks != (n + 127) / 128) return TP_EFORMAT;
+    } else if (k.scheme == TP_FORNM) {
+      if (ncols != 1) return TP_EINVAL;  // decode / decode_sum only
+      if (k.block_size != 128 || k.miniblock_count != 1 || k.num_blocks != (n + 127) / 128) return TP_EFORMAT;
     } else if (rf) {
       if (k.block_size != 512 || k.miniblock_count != 16 || k.num_blocks != (n + 511) / 512) return TP_EFORMAT;
       if (!k.starts1 || !k.data1) return TP_EINVAL;
@@ -1327,7 +1357,8 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
     if (n > 0 && (!k.starts0 || !k.data0)) return TP_EINVAL;
     any_rfor |= rf;
     Col& cc = P.col[c];
-    cc.scheme = k.scheme == TP_FOR ? S_FOR : k.scheme == TP_DFOR ? S_DFOR : k.scheme == TP_RFOR ? S_RFOR : S_NONE;
+    cc.scheme = k.scheme == TP_FOR ? S_FOR : k.scheme == TP_DFOR ? S_DFOR : k.scheme == TP_RFOR ? S_RFOR
+              : k.scheme == TP_FORNM ? S_FORNM : S_NONE;
     cc.nblocks = (uint32_t)k.num_blocks;
     uint32_t rw = 0;
     for (int s = 0; s < (rf ? 2 : 1); ++s) {
@@ -1402,7 +1433,7 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
   // queries hold more per-warp state (3 CTAs/SM at most): a smaller ring keeps them at 3
   // (FOR-only single columns are HBM-bound and get the big ring; DFOR / RFOR decodes are
   // instruction-bound and trade ring space for one more resident CTA)
-  const bool for_only = ncols == 1 && P.col[0].scheme == S_FOR;
+  const bool for_only = ncols == 1 && (P.col[0].scheme == S_FOR || P.col[0].scheme == S_FORNM);
   const uint32_t ring_kb = ncols > 1 ? TP_QUERY_RING_KB : (for_only ? TP_RING_KB : TP_QUERY_RING_KB);
   while (nstg > 2 && (size_t)nstg * P.stage_words * 4 > ring_kb * 1024) --nstg;
   P.nstages = nstg;
@@ -1480,6 +1511,7 @@ tp_status tp_decode_sum(const tp_column* dcol, int64_t* d_sum, void* stream) {
       break;
     case M_DFOR: launch(k_decode_sum<M_DFOR>, smem, cap, stream, P, out); break;
     case M_NONE: launch(k_decode_sum<M_NONE>, smem, cap, stream, P, out); break;
+    case M_FORNM: launch(k_decode_sum<M_FORNM>, smem, cap, stream, P, out); break;
     default: launch(k_decode_sum<M_RFOR>, smem, cap, stream, P, out); break;
   }
   return launched();
@@ -1521,6 +1553,7 @@ tp_status decode_global_impl(const tp_column* dcol, int32_t* d_out, bool raw, vo
   }
   switch (scheme_mask(P)) {
     case M_FOR: launch(k_decode_global<M_FOR>, smem, cap, stream, P, tmap, d_out); break;
+    case M_FORNM: launch(k_decode_global<M_FORNM>, smem, cap, stream, P, tmap, d_out); break;
     case M_DFOR: launch(k_decode_global<M_DFOR>, smem, cap, stream, P, tmap, d_out); break;
     case M_NONE: launch(k_decode_global<M_NONE>, smem, cap, stream, P, tmap, d_out); break;
     default: launch(k_decode_global<M_RFOR>, smem, cap, stream, P, tmap, d_out); break;
@@ -1539,6 +1572,8 @@ tp_status tp_select_project_sum(const tp_column* dcols, int ncols, const int32_t
                                 int a, int b, int64_t* d_result, void* stream) {
   if (!dcols || !lo || !hi || !d_result || ncols < 1 || ncols > TP_MAX_COLS) return TP_EINVAL;
   if (proj_op < TP_PROJ_COL || proj_op > TP_PROJ_COUNT) return TP_EINVAL;
+  for (int c = 0; c < ncols; ++c)
+    if (dcols[c].scheme == TP_FORNM) return TP_EINVAL;  // the ablation format: decode / decode_sum only
   if (proj_op != TP_PROJ_COUNT && (a < 0 || a >= ncols)) return TP_EINVAL;
   if ((proj_op == TP_PROJ_MUL || proj_op == TP_PROJ_SUB) && (b < 0 || b >= ncols)) return TP_EINVAL;
   if (dcols[0].n == 0) return TP_OK;
@@ -1595,6 +1630,8 @@ tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int nc
                         uint64_t* d_counts, uint32_t ngroups, void* stream) {
   if (!dcols || !roles || !d_sums || !d_counts || ncols < 1 || ncols > TP_MAX_COLS || ngroups < 1) return TP_EINVAL;
   if (agg < TP_AGG_SUM || agg > TP_AGG_SUB) return TP_EINVAL;
+  for (int c = 0; c < ncols; ++c)
+    if (dcols[c].scheme == TP_FORNM) return TP_EINVAL;  // the ablation format: decode / decode_sum only
   int nmeas = 0;
   for (int c = 0; c < ncols; ++c) {
     const tp_star_col& r = roles[c];
@@ -1656,7 +1693,7 @@ tp_status tp_plain_sum(const int32_t* d_x, uint64_t n, int64_t* d_sum, void* str
 }
 
 tp_status tp_bitmap_sum(const tp_column* dcol, const uint32_t* d_bitmap, int64_t* d_sum, void* stream) {
-  if (!dcol || !d_bitmap || !d_sum) return TP_EINVAL;
+  if (!dcol || !d_bitmap || !d_sum || dcol->scheme == TP_FORNM) return TP_EINVAL;
   if (dcol->n == 0) return TP_OK;
   Params P;
   size_t smem_unused = 0;

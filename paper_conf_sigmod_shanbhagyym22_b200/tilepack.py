@@ -16,8 +16,9 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("TILEPACK_LIB_OVERRIDE") or os.path.join(_HERE, "libtilepack.so")  # override: A/B builds
 GUARD_WORDS = 4
 
-TP_FOR, TP_DFOR, TP_RFOR, TP_NONE = 1, 2, 3, 4
-SCHEMES = {"for": TP_FOR, "dfor": TP_DFOR, "rfor": TP_RFOR, "none": TP_NONE}
+TP_FOR, TP_DFOR, TP_RFOR, TP_NONE, TP_FORNM = 1, 2, 3, 4, 5
+# "fornm": GPU-FOR without miniblocks, the miniblock ablation (decode / decode_sum only)
+SCHEMES = {"for": TP_FOR, "dfor": TP_DFOR, "rfor": TP_RFOR, "none": TP_NONE, "fornm": TP_FORNM}
 SCHEME_NAMES = {v: k for k, v in SCHEMES.items()}
 TP_PROJ = {"col": 0, "mul": 1, "sub": 2, "count": 3}
 TP_MAX_COLS = 6

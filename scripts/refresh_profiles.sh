@@ -21,3 +21,4 @@ timeout 600 python scripts/bench_random_access.py --reps 5 --out $R/random_acces
 timeout 600 python scripts/bench_cascaded.py --out $R/cascaded.json > $R/cascaded.log 2>&1; echo "cascaded rc=$?"
 timeout 600 python scripts/bench_waterfall.py --out $R/waterfall.json > $R/waterfall.log 2>&1; echo "waterfall rc=$?"
 timeout 900 python scripts/bench_ssb.py --sf 160 --reps 5 --out $R/ssb_sf160.json > $R/ssb160.log 2>&1; echo "ssb160 rc=$?"
+timeout 600 python scripts/bench_nomb.py --out $R/nomb.json > $R/nomb.log 2>&1; echo "nomb rc=$?"

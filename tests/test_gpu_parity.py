@@ -216,3 +216,20 @@ def test_full_size_dfor_rfor(scheme, gen):
     got = tp.decode(d)
     assert torch.equal(got, torch.from_numpy(want).cuda())
     assert int(tp.decode_sum(d).item()) == oracle.column_sum(want)
+
+
+def test_no_miniblock_variant():
+    """the miniblock ablation: GPU decode / decode_sum of GPU-FOR without miniblocks
+    == the oracle's decode, every bitwidth and ragged lengths; query operators refuse it."""
+    for b in (0, 1, 7, 16, 31, 32):
+        _check_column(datagen.uniform_bits(b, 512 * 23 + 45, seed=b), "fornm")
+    for name, x in list(datagen.mixed_columns(seed=31))[::4]:
+        if len(x):
+            _check_column(x, "fornm")
+    rng = np.random.default_rng(5)  # skewed: a few outliers widen a whole block (vs one miniblock)
+    x = rng.integers(0, 2**6, 3_000_017, dtype=np.int64)
+    x[rng.integers(0, len(x), 3000)] = 2**20
+    _check_column(x.astype(np.int32), "fornm")
+    d = tp.encode(x.astype(np.int32), "fornm").to_device()
+    with pytest.raises(tp.TilepackError):
+        tp.select_project_sum([d], [0], [5], "col", 0)

@@ -109,3 +109,18 @@ def test_none_layout():
         assert list(h.starts0[:nb]) == [512 * k for k in range(nb)] and h.starts0[nb] == h.col.words0
         assert np.array_equal(h.data0[:n].view(np.int32), x) and not h.data0[n:].any()
         assert h.nbytes() == 4 * n
+
+
+def test_no_miniblock_variant_byte_identical():
+    """GPU-FOR without miniblocks: the product's host encoder == the oracle's FOR
+    with one 128-entry miniblock per block, byte for byte; size = 4 (3 + nb + 1 + sum(2 + 4 b))."""
+    for name, x in datagen.mixed_columns(seed=9):
+        h = tp.encode(x, "fornm")
+        e = oracle.encode("fornm", x)
+        _same(h, e)
+        assert int(h.col.miniblock_count) == 1
+    for x in datagen.small_alphabet_columns(3):
+        _same(tp.encode(x, "fornm"), oracle.encode("fornm", x))
+    # uniform b bits: every block has width b -> exactly the miniblock format's size
+    x = datagen.uniform_bits(13, 128 * 1000, seed=2)
+    assert tp.encode(x, "fornm").nbytes() == tp.encode(x, "for").nbytes()
