@@ -542,8 +542,12 @@ __device__ __forceinline__ void consumers_sync() {
   asm volatile("bar.sync 1, %0;" ::"n"(CONSUMER_WARPS * 32) : "memory");
 }
 
+#ifndef TP_SPARSE_LANE_MAX
+#define TP_SPARSE_LANE_MAX 8  // ... and (FOR filters / measures) the busiest lane's alive rows
+#endif
 #ifndef TP_SPARSE_MAX
-#define TP_SPARSE_MAX 256  // alive rows (of a warp's 1024) at or below which a column goes sparse
+#define TP_SPARSE_MAX 512  // alive rows (of a warp's 1024) at or below which a column goes sparse
+                           // (512 / 8 measured best over the 13 SSB queries at SF20)
 #endif
 #ifndef TP_QUERY_COMPACT
 #define TP_QUERY_COMPACT true
@@ -786,6 +790,8 @@ struct StarArgs {
   uint32_t gs_off, ws_off;       // per-warp scratch offsets (words) of the group / staged-measure arrays
   uint32_t ht_slots, ht_shift;   // shared-memory aggregation table (grouped queries)
   uint32_t sparse_max;           // warp alive-row count at or below which a column is evaluated sparsely
+  uint32_t sparse_lane_max;      // ... and the busiest lane's alive rows: the sparse loop runs for the
+                                 // warp's maximum (alive rows cluster: runs of an order's lines)
   long long* sums;
   unsigned long long* counts;
 };
@@ -915,7 +921,12 @@ struct StarOp : OpBase {
     const uint32_t lane = g.lane;
     const uint32_t nal = __reduce_add_sync(FULL, __popc(alive));
     const bool sparse =
-        !dfor && (nal <= A->sparse_max || (GROUPED && role == TP_ROLE_MEASURE && !A->mstage[c]));
+        !dfor && ((nal <= A->sparse_max &&
+                   // a FOR filter / measure decodes densely for a few instructions a row: it goes
+                   // sparse only if the busiest lane's rows are few too (probes and RFOR columns
+                   // save far more per skipped row: L2 lookups, run expansion)
+                   (role == TP_ROLE_PROBE || rfor || __reduce_max_sync(FULL, __popc(alive)) <= A->sparse_lane_max)) ||
+                  (GROUPED && role == TP_ROLE_MEASURE && !A->mstage[c]));
     RforChunk k;
     uint32_t carry = 0u;
     if (rfor) {
@@ -1660,6 +1671,8 @@ tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int nc
   A.agg = agg;
   A.ngroups = ngroups;
   A.sparse_max = TP_SPARSE_MAX;
+  A.sparse_lane_max = TP_SPARSE_LANE_MAX;
+  if (const char* e = getenv("TILEPACK_SPARSE_LANE_MAX")) A.sparse_lane_max = (uint32_t)atoi(e);  // tuning
   if (const char* e = getenv("TILEPACK_SPARSE_MAX")) A.sparse_max = (uint32_t)atoi(e);  // tests: force a mode
   const uint32_t hts = grouped ? ht_slots(ngroups) : 0u;
   const uint32_t gwords = grouped ? 32u * 32u : 0u, wwords = nmeas == 2 ? 32u * 32u : 0u;

@@ -95,6 +95,7 @@ def test_gpu_star_query_modes(mode, monkeypatch):
     from paper_conf_sigmod_shanbhagyym22_b200 import tilepack as tp
     if mode != "auto":
         monkeypatch.setenv("TILEPACK_SPARSE_MAX", "0" if mode == "dense" else "1024")
+        monkeypatch.setenv("TILEPACK_SPARSE_LANE_MAX", "0" if mode == "dense" else "32")
     for seed in (1, 2):
         d = _inputs(seed)
         dev = {}
