@@ -24,10 +24,9 @@ def main():
 
 All numbers on one B200 (148 SMs, sm_100a, SM clock {b['clocks']['sm_mhz']:.0f} MHz under load = max, no throttle
 reasons recorded), CUDA 12.9, driver 580.  Roofline denominator: `MEASURED_PEAKS.json` `hbm_gbs`
-(copy, read+write; "of measured").  The files below come from `scripts/refresh_profiles.sh`
-(all measurements + ncu captures on one box); the suite, SSB and miniblock files were re-measured
-after later kernel changes (their commits say which).  This README is generated from them by
-`scripts/profiles_readme.py`.
+(copy, read+write; "of measured").  Every file below comes from ONE run of
+`scripts/refresh_profiles.sh` (all measurements + ncu captures on one box, at the final commit of
+round 1); this README is generated from them by `scripts/profiles_readme.py`.
 
 | file | what |
 |---|---|
