@@ -124,3 +124,20 @@ def test_no_miniblock_variant_byte_identical():
     # uniform b bits: every block has width b -> exactly the miniblock format's size
     x = datagen.uniform_bits(13, 128 * 1000, seed=2)
     assert tp.encode(x, "fornm").nbytes() == tp.encode(x, "for").nbytes()
+
+
+def test_gpu_encode_bound_covers_every_encoding():
+    """tp_gpu_encode_bound (host arithmetic): a capacity that always suffices -- never below the
+    words the encoder actually produces (worst case: every miniblock 32 bits wide / every row its
+    own run), equal to it for full-range data; the workspace grows with the chunk count."""
+    cols = [datagen.uniform_bits(32, 5000 + 77, seed=1), datagen.runs(9000, 1, seed=2),
+            np.zeros(1, np.int32), datagen.uniform_bits(7, 512 * 9, seed=3)]
+    for x in cols:
+        for s in ("for", "dfor", "rfor", "none"):
+            sc = tp.SCHEMES[s]
+            nb, w0, w1 = tp.tp_gpu_encode_bound(sc, len(x))
+            h = tp.encode(x, s)
+            assert nb == h.col.num_blocks and w0 >= h.col.words0 and w1 >= h.col.words1, (s, len(x))
+    x = datagen.uniform_bits(32, 128 * 40, seed=4)
+    assert tp.tp_gpu_encode_bound(tp.TP_FOR, len(x))[1] == tp.encode(x, "for").col.words0
+    assert tp.tp_gpu_encode_workspace_bytes(10**8) > tp.tp_gpu_encode_workspace_bytes(10**6) > 0
