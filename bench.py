@@ -1,21 +1,34 @@
 #!/usr/bin/env python
-"""bench.py -- BASELINE.json config 2 (GPU-FOR decode-only on a 500M-entry int32 column)
-through the tilepack C ABI on B200, plus the oracle timed on the host as cpu_baseline.
+"""bench.py -- BASELINE.json's metric on B200 through the tilepack C ABI: decoded GB/s and % of the
+HBM roofline per scheme, SSB query ms; the oracle timed on the host beside it (cpu_baseline).
 
-Step = one pass of the decode hot path over the whole column: tile addressing, TMA
-staging, header + miniblock offsets, bit unpack, consume in registers (fused int64 sum)
--- SURVEY.md 8(a) rows a1-a4, a7 -- plus, for N > 1, the NCCL allreduce of the
-partial aggregate (row a9).  Default workload: U[0, 2^16), the paper's E1 column
-(P:720-724, 500 million values), i.e. the b = 16 point of the bitwidth sweep;
---bits picks another point, --sweep adds the whole 0..32 sweep as an extra object.
+Headline `value` (the driver's scaling number): BASELINE config 2 at the paper's E1 point --
+GPU-FOR decode-only on a 500M-entry U[0,2^16) int32 column, the decode fused into an
+int64 sum.  A step = one pass of the decode hot path over the column: tile addressing, TMA
+staging, headers + miniblock offsets, bit unpack, consume in registers (SURVEY.md 8(a) rows
+a1-a4, a7) + for N > 1 the NCCL allreduce of the partial aggregate (a9).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--bits B] [--sweep] [--impl reference]
+Extra objects on the same line (each with its own parity check against the plain definition):
+  schemes   -- BASELINE configs 2-4 at 500M rows on GPU 0: FOR b=4 (issue-bound) and b=16, DFOR D1
+               (config 3), RFOR runs of 4 (config 4): decode->sum and decode->global
+               kernel ms (median of 5, L2 flushed), HBM fraction, instructions / value and issue
+               fraction from the committed ncu profile, decoded column == x, sum == sum(x)
+  issue_roof-- the measured INT32 issue roof: SHF/LOP3/IADD3/IMAD throughput
+  ssb_sf20  -- BASELINE config 5: the 13 SSB queries at SF 20 with inline decompression, tile-range
+               shards of lineorder per rank (rank-local generation), one fused star kernel + one
+               allreduce per query; ms (max over ranks), HBM floor fraction, results == the
+               oracle's answers (tests/golden/ssb_sf20.json, written by scripts/make_ssb_golden.py)
+  cpu_baseline -- the oracle (oracle/oracle.c, Alg. 1 per entry) decoding + summing the same
+               encoded column on ALL host cores (tile-range threads), plus its 1-core figure
+  config1   -- BASELINE config 1: the oracle's round trip of 1M-row columns at b = 1..16, seconds
 
-Multi-GPU: one process per GPU (torchrun), each rank owns its own 500M column (weak
-scaling: tile-range partitions of a dataset N x larger), partial sums combined with
-one NCCL allreduce per step.  Timing: CUDA events on the launch stream, barrier +
-synchronize on both sides, max over ranks.  L2: the compressed column (>= 1 GB at
-b=16) is 8x the 126 MB L2, so consecutive steps never hit L2 (no flush needed).
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--bits B] [--quick] [--impl reference]
+
+Multi-GPU: one process per GPU (torchrun); the headline is weak scaling (each rank decodes its own
+500M-row tile range of an N x 500M logical column, "scaling": "weak"), the SSB leg is strong
+scaling (SF 20 split by 512-row tile ranges).  Timing: CUDA events on the launch stream, barrier +
+synchronize on both sides, max over ranks.  L2: the compressed column (1.05 GB at b=16) is 8x the
+126 MB L2, so consecutive steps never hit L2; the extra legs flush L2 before every rep.
 """
 from __future__ import annotations
 
@@ -23,6 +36,7 @@ import argparse
 import json
 import os
 import statistics
+import subprocess
 import sys
 import threading
 import time
@@ -34,19 +48,23 @@ sys.path.insert(0, ROOT)
 
 N_ROWS = 500_000_000
 PAPER_DECODED_GBS = 2e9 / 1.55e-3 / 1e9  # V100, D=16, 500M U(0,2^16): 1.55 ms -> 1290 GB/s
+METRIC = "decoded GB/s (GPU-FOR decode-only, fused int64 sum)"
 
 
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=500)
+    ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--bits", type=int, default=16)
     ap.add_argument("--rows", type=int, default=N_ROWS)
-    ap.add_argument("--sweep", action="store_true", help="also time every bitwidth 0..32 (extra object)")
     ap.add_argument("--impl", default="tilepack", choices=["tilepack", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--quick", action="store_true", help="headline only (no extra legs, no cpu baseline)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-ssb", action="store_true")
+    ap.add_argument("--no-schemes", action="store_true")
+    ap.add_argument("--ssb-sf", type=float, default=20)
     return ap.parse_args()
 
 
@@ -59,7 +77,10 @@ def dist_env():
 
 # ------------------------------------------------------------------ clocks (NVML, during the timed region)
 class ClockSampler:
-    def __init__(self, index: int, period: float = 0.005):
+    """Samples the SM clock and the clock-event reasons back to back (no sleep: an NVML query
+    takes ~0.1 ms, so even a few-ms timed region yields tens of samples)."""
+
+    def __init__(self, index: int, period: float = 0.0):
         self.samples, self.reasons, self.max_mhz = [], set(), None
         self.period, self._stop = period, threading.Event()
         try:
@@ -81,16 +102,18 @@ class ClockSampler:
                 self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
                 r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
                 for bit, name in self._NAMES.items():
-                    if r & bit and name != "gpu_idle":
+                    if r & bit and name not in ("gpu_idle", "applications_clocks_setting"):
                         self.reasons.add(name)
             except Exception:
                 pass
-            time.sleep(self.period)
+            if self.period:
+                time.sleep(self.period)
 
     def __enter__(self):
         if self.nv:
             self.t = threading.Thread(target=self._run, daemon=True)
             self.t.start()
+            time.sleep(0.002)  # the sampler is running before the timed region starts
         return self
 
     def __exit__(self, *a):
@@ -101,7 +124,7 @@ class ClockSampler:
     def summary(self):
         return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
                 "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples),
-                "source": "NVML (same counters as nvidia-smi), sampled every 5 ms during the timed steps"}
+                "source": "NVML (same counters as nvidia-smi), sampled back to back during the timed steps"}
 
 
 def measured_peak():
@@ -112,70 +135,266 @@ def measured_peak():
         return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
+def _profile(name):
+    try:
+        return json.load(open(os.path.join(ROOT, "profiles", name)))
+    except Exception:
+        return None
+
+
 def ncu_traffic(workload: str):
     """dram bytes per launch of the dominant kernel from the committed ncu --set full summary."""
+    prof = _profile("ncu_summary.json")
     try:
-        prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_summary.json")))
         t = prof["kernels"][workload]
         return int(t["dram_bytes_read"]) + int(t["dram_bytes_write"])
     except Exception:
         return None
 
 
+def cpu_model():
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return None
+
+
 # ------------------------------------------------------------------ workload
 def make_column(bits: int, rows: int, rank: int):
     import datagen
-    seed = 2000 + bits + 1000 * rank
-    return datagen.uniform_bits(bits, rows, seed=seed)
+    return datagen.uniform_bits(bits, rows, seed=2000 + bits + 1000 * rank)
 
 
-def cpu_baseline(h, rows: int, budget_rows: int = N_ROWS):
-    """The oracle (oracle/, single-threaded scalar C, Algorithm 1 per entry) decoding and
-    summing a bounded sample: the first `budget_rows` rows of the same encoded column."""
+def _oracle_encoded(h):
     import oracle
-    sample = min(rows, budget_rows)
-    e = oracle.Encoded(scheme="for", header=h.header(), starts=h.starts0[: h.col.num_blocks + 1],
-                       data=h.data0[: h.col.words0])
+    return oracle.Encoded(scheme="for", header=h.header(), starts=h.starts0[: h.col.num_blocks + 1],
+                          data=h.data0[: h.col.words0])
+
+
+def cpu_baseline(h, rows: int):
+    """The oracle (oracle/oracle.c: Algorithm 1 per entry, then the int64 sum) decoding the same
+    encoded column, (a) on 1 core over a bounded 50M-row sample and (b) on ALL host cores over
+    the whole column -- tile-range threads around the unchanged scalar decode (the ctypes call
+    releases the GIL; tiles are independent)."""
+    import oracle
+    from concurrent.futures import ThreadPoolExecutor
+    e = _oracle_encoded(h)
+    one = min(rows, 50_000_000)
     t = time.perf_counter()
-    y = oracle.for_decode_range(e, 0, sample, h.data0)
-    s = oracle.column_sum(y)
-    dt = time.perf_counter() - t
-    return {"value": 4 * sample / dt / 1e9, "unit": "decoded GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"first {sample:,} rows of the same encoded column: Alg. 1 decode per entry + int64 sum "
-                      f"(oracle/oracle.c, 1 thread), {dt:.1f} s", "checksum": int(s)}
+    s1 = oracle.column_sum(oracle.for_decode_range(e, 0, one, h.data0))
+    dt1 = time.perf_counter() - t
+    cores = os.cpu_count() or 1
+    tiles = (rows + 511) // 512
+    bounds = [512 * (tiles * i // cores) for i in range(cores)] + [rows]
+
+    def part(i):
+        lo, hi = bounds[i], min(bounds[i + 1], rows)
+        return oracle.column_sum(oracle.for_decode_range(e, lo, hi, h.data0)) if hi > lo else 0
+
+    t = time.perf_counter()
+    with ThreadPoolExecutor(max_workers=cores) as ex:
+        total = sum(ex.map(part, range(cores)))
+    dtn = time.perf_counter() - t
+    return {"value": 4 * rows / dtn / 1e9, "unit": "decoded GB/s", "cores": cores, "kind": "oracle",
+            "sample": f"all {rows:,} rows of the same encoded column on {cores} threads (tile ranges): Alg. 1 "
+                      f"decode per entry + int64 sum (oracle/oracle.c), {dtn:.2f} s",
+            "cpu_model": cpu_model(), "checksum": int(total),
+            "one_core": {"value": 4 * one / dt1 / 1e9, "unit": "decoded GB/s", "cores": 1,
+                         "sample": f"first {one:,} rows, {dt1:.2f} s", "checksum": int(s1)}}
+
+
+def config1_oracle():
+    """BASELINE config 1: GPU-FOR round trip of 1M uniform int32 columns, b = 1..16, on the oracle
+    (1 core): seconds for encode + decode of all 16 columns, each decode == x."""
+    import datagen
+    import oracle
+    t = time.perf_counter()
+    ok = True
+    for b in range(1, 17):
+        x = datagen.c1_column(b)
+        e = oracle.for_encode(x)
+        ok &= bool(np.array_equal(oracle.for_decode(e), x))
+    return {"seconds": time.perf_counter() - t, "columns": 16, "rows_each": 1_000_000, "roundtrip_ok": ok,
+            "what": "oracle.for_encode + oracle.for_decode (plain C, 1 core), b = 1..16"}
 
 
 def run_reference(args):
-    """--impl reference: the oracle as it stands on the host cores, same metric/config."""
+    """--impl reference: the oracle as it stands (oracle.encode + Alg. 1 decode + sum) on the host
+    cores, same metric and config, bounded sample per step."""
     rank, world, _ = dist_env()
     if rank != 0:
         return
     import oracle
-    from paper_conf_sigmod_shanbhagyym22_b200 import tilepack as tp  # host encoder only (no GPU call)
-    x = make_column(args.bits, args.rows, 0)
-    h = tp.encode(x, "for")
     sample = min(args.rows, 25_000_000)
-    e = oracle.Encoded(scheme="for", header=h.header(), starts=h.starts0[: h.col.num_blocks + 1],
-                       data=h.data0[: h.col.words0])
+    x = make_column(args.bits, sample, 0)  # the first `sample` rows of the bench column
+    e = oracle.encode("for", x)
+    dg = e.guarded("data")
     for _ in range(args.warmup):
-        oracle.column_sum(oracle.for_decode_range(e, 0, min(sample, 1_000_000), h.data0))
+        oracle.column_sum(oracle.for_decode_range(e, 0, min(sample, 1_000_000), dg))
     times = []
-    for _ in range(args.steps if args.steps <= 20 else 20):
+    for _ in range(min(args.steps, 20)):
         t = time.perf_counter()
-        oracle.column_sum(oracle.for_decode_range(e, 0, sample, h.data0))
+        oracle.column_sum(oracle.for_decode_range(e, 0, sample, dg))
         times.append(time.perf_counter() - t)
     ms = 1e3 * sum(times) / len(times)
     value = 4 * sample / (ms / 1e3) / 1e9
-    line = {"impl": "reference", "metric": "decoded GB/s (GPU-FOR decode-only, fused int64 sum)", "value": value,
-            "unit": "GB/s", "n_gpus": world, "steps": len(times), "warmup": args.warmup, "ms_per_step": ms,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
-            "data": "synthetic",
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world,
+            "steps": len(times), "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {"workload": f"C2 GPU-FOR b={args.bits} U[0,2^{args.bits}) {args.rows:,} rows, decode->sum",
                        "sample_rows_per_step": sample},
             "cpu_baseline": {"value": value, "unit": "GB/s", "cores": 1, "kind": "oracle",
-                             "sample": f"first {sample:,} rows per step, Alg. 1 per entry, 1 thread"},
+                             "sample": f"first {sample:,} rows per step: oracle.encode (once), then Alg. 1 per "
+                                       "entry + int64 sum, 1 thread"},
             "e2e": {"value": value, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ extra legs
+def _timed(torch, stream, fn, flush, reps=5):
+    for _ in range(2):
+        fn()
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(reps):
+        flush.zero_()  # 512 MB > L2 written, then read (the dirty lines are written back before the
+        flush.sum()    # timed launch, which then starts with an L2 of clean, unrelated lines)
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        fn()
+        b.record(stream)
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b))
+    return statistics.median(ts)
+
+
+def scheme_leg(args, tp, dev, stream, torch, roof):
+    """BASELINE configs 2-4 at full size: decode->sum and decode->global per scheme."""
+    import datagen
+    peak, _ = measured_peak()
+    prof = (_profile("r02_issue.json") or {}).get("configs", {})
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    acc = torch.zeros(1, dtype=torch.int64, device=dev)
+    rows = args.rows
+    alu = roof.get("SHF+LOP3+IADD3 (ALU pipe)", {}).get("warp_insts_per_s") if roof else None
+    issue = roof.get("LOP3+IMAD (ALU+FMA pipes)", {}).get("warp_insts_per_s") if roof else None
+    cfgs = [("for_b4", "for", lambda: datagen.uniform_bits(4, rows, seed=2004)),
+            ("for_b16", "for", lambda: datagen.uniform_bits(16, rows, seed=2016)),
+            ("dfor_d1", "dfor", lambda: datagen.d1_sorted(rows, 2**28)),
+            ("rfor_runs4", "rfor", lambda: datagen.runs(rows, 4))]
+    out = {}
+    for name, scheme, gen in cfgs:
+        x = gen()
+        h = tp.encode(x, scheme)
+        d = h.to_device(dev)
+        cb = h.nbytes()
+        truth = int(x.astype(np.int64).sum())
+
+        def do_sum():
+            acc.zero_()
+            tp.tp_decode_sum(d.col, acc, stream)
+        ms_sum = _timed(torch, stream, do_sum, flush)
+        sum_ok = int(acc.item()) == truth
+        dec = torch.empty(rows, dtype=torch.int32, device=dev)
+        ms_g = _timed(torch, stream, lambda: tp.tp_decode(d.col, dec, stream), flush)
+        xd = torch.from_numpy(x).to(dev)
+        glob_ok = bool(torch.equal(dec, xd))
+        r = {"scheme": scheme, "rows": rows, "compressed_bytes": cb, "bits_per_int": 8 * cb / rows,
+             "sum_ms": ms_sum, "sum_decoded_gbs": 4 * rows / ms_sum / 1e6,
+             "sum_hbm_frac": cb / ms_sum / 1e6 / peak,
+             "global_ms": ms_g, "global_decoded_gbs": 4 * rows / ms_g / 1e6,
+             "global_hbm_frac": (cb + 4 * rows) / ms_g / 1e6 / peak,
+             "parity": {"sum_eq_int64_sum_of_x": sum_ok, "decoded_eq_x": glob_ok}}
+        p = prof.get(name)
+        if p:  # instructions per value from the committed ncu capture of the same configuration
+            for mode in ("sum", "global"):
+                if f"{mode}_warp_insts" in p:
+                    wi = p[f"{mode}_warp_insts"]
+                    ms = r[f"{mode}_ms"]
+                    r[f"{mode}_insts_per_value"] = 32 * wi / rows
+                    if issue:
+                        r[f"{mode}_issue_frac"] = wi / (ms / 1e3) / issue
+                    if alu:
+                        r[f"{mode}_alu_roof_frac"] = wi / (ms / 1e3) / alu
+        out[name] = r
+        del d, h, x, dec, xd
+        torch.cuda.empty_cache()
+    return out
+
+
+def ssb_leg(args, tp, dev, stream, torch, rank, world):
+    """BASELINE config 5 at SF 20: 13 queries, tile-range shards per rank, one allreduce per query."""
+    import torch.distributed as dist
+    import datagen.ssb as gen
+    from paper_conf_sigmod_shanbhagyym22_b200.dist import tile_range
+    from paper_conf_sigmod_shanbhagyym22_b200.ssb import QUERIES, SSBEngine
+    peak, _ = measured_peak()
+    total = gen.num_rows(args.ssb_sf)
+    r0, r1 = tile_range(total, rank, world)
+    db = gen.generate(args.ssb_sf, seed=5000, columns=gen.QUERY_COLUMNS, rows=(r0, r1))
+    eng = SSBEngine(db, dev)
+    golden = None
+    sfn = ("%g" % args.ssb_sf).replace(".", "_")
+    gp = os.path.join(ROOT, "tests", "golden", f"ssb_sf{sfn}.json")
+    if os.path.exists(gp):
+        golden = json.load(open(gp))
+        if golden.get("rows") != total:
+            golden = None
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    res = {}
+    for q in QUERIES:
+        prep = eng.prepare(q)
+        cols = sorted({c[0] for c in prep["plan"]["cols"]})
+        cb = sum(eng.host[c].nbytes() for c in cols)
+        sums = torch.zeros(prep["ngroups"], dtype=torch.int64, device=dev)
+        counts = torch.zeros_like(sums)
+        kt, qt = [], []
+        for it in range(7):
+            sums.zero_()
+            counts.zero_()
+            flush.zero_()
+            flush.sum()
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+            e0.record(stream)
+            eng.execute(prep, sums, counts, stream)
+            e1.record(stream)
+            if world > 1:
+                dist.all_reduce(sums)
+                dist.all_reduce(counts)
+            e2.record(stream)
+            torch.cuda.synchronize()
+            if it >= 2:
+                kt.append(e0.elapsed_time(e1))
+                qt.append(e0.elapsed_time(e2))
+        t = torch.tensor([statistics.median(kt), statistics.median(qt), float(cb)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        kms, qms, cbmax = (float(v) for v in t.tolist())
+        r = {"query_ms": qms, "kernel_ms": kms, "compressed_bytes_per_gpu_max": int(cbmax),
+             "hbm_floor_ms": cbmax / peak / 1e6, "hbm_frac": cbmax / (kms / 1e3) / 1e9 / peak}
+        if rank == 0 and golden is not None:
+            got = eng.result(q, prep, sums, counts)
+            r["parity"] = [list(g) for g in got] == golden["results"][q]
+        res[q] = r
+    geo = float(np.exp(np.mean([np.log(v["query_ms"]) for v in res.values()])))
+    out = {"sf": args.ssb_sf, "rows": total, "rows_per_gpu": r1 - r0, "n_gpus": world, "geomean_query_ms": geo,
+           "geomean_hbm_frac": float(np.exp(np.mean([np.log(v["hbm_frac"]) for v in res.values()]))),
+           "scaling": "strong (fixed SF, lineorder split by 512-row tile ranges)",
+           "timing": "median of 5 after 2 warm-ups, L2 flushed, CUDA events; query_ms = star kernel + allreduce, "
+                     "max over ranks; dimension lookup tables built once per query outside the timed region",
+           "parity_reference": os.path.relpath(gp, ROOT) if golden else None,
+           "parity_all": all(v.get("parity", False) for v in res.values()) if golden and rank == 0 else None,
+           "queries": res}
+    del eng
+    torch.cuda.empty_cache()
+    return out
 
 
 def main():
@@ -253,6 +472,7 @@ def main():
     k_avg = sum(k_ms) / len(k_ms)
     peak, peak_src = measured_peak()
     achieved = comp_bytes / (k_avg / 1e3) / 1e9
+    assert tp.tp_device_errors(stream) == 0
 
     # ---------------- e2e: host buffers through the C ABI, H2D + decode + D2H inside the timed region
     pin = {k: torch.from_numpy(v.view(np.int32)).pin_memory() for k, v in
@@ -290,6 +510,7 @@ def main():
     if world > 1:
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
     e2e_ms = float(te.item())
+    del dst, pin
 
     # ---------------- the "None" roof (uncompressed int32 read of the same consumer), rank-local
     none_gbs = None
@@ -308,14 +529,19 @@ def main():
     except Exception:
         pass
 
-    sweep = None
-    if args.sweep:
-        sweep = run_sweep(args, tp, dev, stream, torch)
+    extra = {}
+    if not args.quick:
+        roof = tp.measure_int_roof() if rank == 0 else None
+        extra["issue_roof"] = roof
+        if world == 1 and not args.no_schemes:
+            extra["schemes"] = scheme_leg(args, tp, dev, stream, torch, roof)
+        if not args.no_ssb:
+            extra[("ssb_sf%g" % args.ssb_sf).replace(".", "_")] = ssb_leg(args, tp, dev, stream, torch, rank, world)
 
     if rank == 0:
         sms, occ = tp.tp_device_info()
         line = {
-            "metric": "decoded GB/s (GPU-FOR decode-only, fused int64 sum)",
+            "metric": METRIC,
             "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": value / PAPER_DECODED_GBS if world == 1 else None,
@@ -324,7 +550,8 @@ def main():
                                    "decode fused into int64 sum (paper E1, P:720-724)",
                        "rows_per_gpu": args.rows, "bits": args.bits, "compressed_bytes_per_gpu": comp_bytes,
                        "bits_per_int": 8 * comp_bytes / args.rows,
-                       "l2": "inputs larger than L2 (compressed column > 8x 126 MB), no flush",
+                       "l2": "inputs larger than L2 (compressed column > 8x 126 MB), no flush in the headline; "
+                             "the extra legs flush L2 (512 MB write) before every rep",
                        "grid": f"{sms} SMs x {occ} CTAs, 160 threads (1 TMA producer warp + 4 consumer warps)",
                        "parallelism": f"tile-range partitions, {world} GPU(s), NCCL allreduce of the partial sum"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -338,50 +565,16 @@ def main():
             "clocks": clk.summary(),
             "context": {"paper_v100_decoded_gbs": PAPER_DECODED_GBS,
                         "none_uncompressed_read_gbs": none_gbs,
-                        "host_encode_s": enc_s, "setup_s": time.perf_counter() - t_setup},
+                        "host_encode_s": enc_s},
         }
-        if sweep is not None:
-            line["sweep"] = sweep
-        if world == 1 and not args.no_cpu_baseline:
+        line.update(extra)
+        if world == 1 and not args.quick and not args.no_cpu_baseline:
             line["cpu_baseline"] = cpu_baseline(h, args.rows)
+            line["config1"] = config1_oracle()
+        line["context"]["setup_and_legs_s"] = time.perf_counter() - t_setup
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
-
-
-def run_sweep(args, tp, dev, stream, torch):
-    """Bitwidth sweep 0..32 (BASELINE config 2): per-b kernel time, decoded + compressed GB/s."""
-    peak, _ = measured_peak()
-    out = {}
-    acc = torch.zeros(1, dtype=torch.int64, device=dev)
-    for b in range(33):
-        x = make_column(b, args.rows, 0)
-        h = tp.encode(x, "for")
-        d = h.to_device(dev)
-        truth = int(x.astype(np.int64).sum())
-        del x
-        for _ in range(3):
-            acc.zero_()
-            tp.tp_decode_sum(d.col, acc, stream)
-        torch.cuda.synchronize()
-        assert int(acc.item()) == truth
-        flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
-        ts = []
-        for _ in range(10):
-            flush.sum()  # L2 flush by reading (no dirty lines to write back)
-            a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            a.record(stream)
-            tp.tp_decode_sum(d.col, acc, stream)
-            e.record(stream)
-            torch.cuda.synchronize()
-            ts.append(a.elapsed_time(e))
-        ms = statistics.median(ts)
-        cb = h.nbytes()
-        out[str(b)] = {"ms": ms, "decoded_gbs": 4 * args.rows / ms / 1e6, "compressed_gbs": cb / ms / 1e6,
-                       "hbm_frac": cb / ms / 1e6 / peak, "bits_per_int": 8 * cb / args.rows}
-        del d, h, flush
-        torch.cuda.empty_cache()
-    return out
 
 
 if __name__ == "__main__":

@@ -77,8 +77,10 @@ typedef enum {
  *   RFOR:     starts0/data0 = value stream, starts1/data1 = run-length stream,
  *             one stream block per 512-row block (R17).
  *   max_tile_words0/1: largest word span of one 512-row tile in stream 0/1
- *             (filled by tp_encode / tp_shard; 0 = unknown, the decoder then
- *             assumes the format's worst case).  Sizes the shared-memory ring.
+ *             (filled by tp_encode / tp_gpu_encode / tp_shard / tp_validate;
+ *             0 = unknown, the decoder then assumes the format's worst case).
+ *             Sizes the shared-memory ring; a value below the column's real
+ *             span is detected on the device (TP_DEVERR_TILE_WORDS).
  */
 typedef struct {
   uint32_t scheme;            /* tp_scheme                                      */
@@ -130,7 +132,34 @@ uint64_t tp_compressed_bytes(const tp_column* col);
 tp_status tp_shard(const tp_column* host_col, uint64_t row_lo, uint64_t row_hi,
                    uint32_t* rebased0, uint32_t* rebased1, tp_column* view);
 
+/* Format check of a HOST column (R1-R19): header fields
+ * (block_size / miniblock_count / num_blocks of the scheme), block_starts
+ * non-decreasing and ending at words0 (words1), every bitwidth byte <= 32
+ * (R3, R5) with the unused bytes zero, every block exactly 2 + sum of its
+ * miniblock widths words (Alg. 1 lines 13-14; FORNM 2 + 4 b;
+ * RFOR 6 + its tight miniblocks, R17), RFOR run counts in [1, rows of the
+ * block] and equal in both streams.  Returns TP_EFORMAT at the first
+ * violation, TP_OK otherwise, and writes the column's exact largest tile
+ * span per stream (the value max_tile_words0/1 must not be below) to
+ * *max_tile_words0 / *max_tile_words1 (either may be NULL).  O(num_blocks)
+ * reads, single-threaded; the device calls do NOT run it (they trust the
+ * bytes -- see tp_device_errors for what they do check). */
+tp_status tp_validate(const tp_column* host_col, uint32_t* max_tile_words0, uint32_t* max_tile_words1);
+
 /* ---------------------------------------------------------------- device */
+
+/* Format violations the DEVICE calls detect while they run (bit flags; the kernel
+ * stays inside its buffers -- a bitwidth byte > 32 is used as 32, a tile range longer
+ * than the ring region sized from max_tile_words is copied only up to the region -- and
+ * the affected results are undefined):
+ *   TP_DEVERR_BITWIDTH   a miniblock bitwidth byte > 32 (R3, R5)
+ *   TP_DEVERR_TILE_WORDS a tile range spans more words than max_tile_words0/1 says
+ *   TP_DEVERR_RUNS       an RFOR stream block counts more than 512 runs (R17)
+ * tp_device_errors synchronizes `stream`, writes the flags accumulated by this
+ * library's kernels on the current device since the last call to *flags (host), and
+ * clears them.  Returns TP_ECUDA if the synchronisation or the read fails. */
+enum { TP_DEVERR_BITWIDTH = 1, TP_DEVERR_TILE_WORDS = 2, TP_DEVERR_RUNS = 4 };
+tp_status tp_device_errors(uint32_t* flags, void* stream);
 
 /* Decode the whole DEVICE column into d_out[0..n) (int32, device).
  * One pass over HBM: each 512-row tile is staged once into shared memory by
@@ -243,7 +272,8 @@ tp_status tp_decode_cascaded(const tp_column* dcol, int32_t* d_out, uint32_t* d_
  * The paper compresses once on the host; every 512-row tile is encoded
  * independently, so the encoder also runs on the GPU
  * in one pass over a DEVICE column: warps plan and pack tiles, a decoupled look-back over
- * 4096-row chunks gives each tile its word offset.  The bytes are
+ * chunks (16384 rows for FOR / DFOR, 8192 for RFOR) gives each tile its word offset
+ * (SURVEY.md NEXT-3).  The bytes are
  * identical to tp_encode's.  d_x must be 16-byte aligned.
  *
  * d_work: DEVICE scratch of tp_gpu_encode_workspace_bytes(n) bytes (8-byte aligned), owned
@@ -283,6 +313,17 @@ tp_status tp_gpu_encode_result(int scheme, uint64_t n, const uint32_t* d_starts0
 tp_status tp_gpu_encode(int scheme, const int32_t* d_x, uint64_t n, uint32_t* d_starts0, uint32_t* d_data0,
                         uint64_t cap0, uint32_t* d_starts1, uint32_t* d_data1, uint64_t cap1, void* d_work,
                         tp_column* out, void* stream);
+
+/* ---------------------------------------------- measurement (not the method)
+ * The INT32 issue roof of SURVEY.md 8(d): the low-bitwidth decoders are bound by
+ * integer instruction issue, not HBM (P:1705-1707 for DFOR on the paper's GPU).
+ * Launches one microbenchmark kernel on every SM (8 CTAs x 256 threads, 8 independent
+ * dependency chains per thread) asynchronously on `stream`; *warp_insts (host) = the
+ * warp instructions of the measured kind it executes (the caller times the launch).
+ * kind: 0 SHF, 1 LOP3, 2 IADD3, 3 IMAD, 4 SHF / LOP3 / IADD3 mix (ALU pipe only: the
+ * unpack-and-sum mix), 5 LOP3 / IMAD alternating (ALU + FMA pipes: the per-SMSP issue
+ * limit).  d_sink: one DEVICE u32 (practically never written). */
+tp_status tp_bench_int_roof(int kind, uint32_t iters, uint32_t* d_sink, uint64_t* warp_insts, void* stream);
 
 /* --------------------------------------------------------------- utility */
 

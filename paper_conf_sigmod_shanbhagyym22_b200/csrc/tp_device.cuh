@@ -136,6 +136,20 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
+// ------------------------------------------------------------------ format-violation flags
+// (include/tilepack.h tp_device_errors; one copy per translation unit -- the pipeline
+// kernels' copy in tp_kernels.cu is the one the ABI reads)
+static __device__ uint32_t g_tp_err;
+static __device__ __noinline__ void tp_flag_error(uint32_t bit) { atomicOr(&g_tp_err, bit); }
+// a miniblock bitwidth byte: > 32 is a format violation (R3, R5), used as 32
+__device__ __forceinline__ uint32_t checked_bw(uint32_t b) {
+  if (b > 32u) {
+    tp_flag_error(1u);  // TP_DEVERR_BITWIDTH
+    b = 32u;
+  }
+  return b;
+}
+
 // ------------------------------------------------------------------ column params
 // One stream of an encoded column as the kernels see it (host fills).
 enum : uint32_t { K_FOR = 0, K_DFOR = 1, K_RFOR = 2, K_NONE = 3 };  // stream kinds
@@ -146,6 +160,7 @@ struct Stream {
   uint32_t starts_off;  // word offset of this stream's block_starts region
   uint32_t kind;        // K_FOR / K_DFOR: 4 blocks per tile; K_RFOR: 1 stream block per tile
   uint32_t nblocks;
+  uint32_t data_cap;    // bytes of the stage's data region (TP_DEVERR_TILE_WORDS beyond it)
 };
 struct Col {
   uint32_t scheme;      // S_FOR / S_DFOR / S_RFOR
@@ -352,7 +367,7 @@ __device__ __forceinline__ MbView for_view(const uint32_t* sd, const uint32_t* s
     const uint32_t* blk = sd + (bs - lo + dshift);
     v.ref = blk[0];                                 // reference (Alg. 1 line 3)
     const uint32_t bw = blk[1];                     // bitwidth word (line 6)
-    v.b = min((bw >> (8u * j)) & 255u, 32u);        // line 11
+    v.b = checked_bw((bw >> (8u * j)) & 255u);      // line 11
     v.w = blk + 2u + bw_prefix(bw, j);              // lines 13-14 (header_offset = 2)
   } else {
     v.ref = 0u; v.b = 0u; v.w = sd;

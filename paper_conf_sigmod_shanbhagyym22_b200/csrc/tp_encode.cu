@@ -6,8 +6,10 @@
 // every 512-row tile is encoded independently, so the only
 // cross-tile dependency is the word offset of each tile in the output -- an exclusive prefix
 // sum of tile sizes.  One pass over HBM:
-//   * persistent CTAs of 8 warps take 8-tile chunks (4096 rows) in order from an atomic
-//     counter; warp w loads tile w of the chunk (coalesced 16-byte loads) into shared memory;
+//   * persistent CTAs of 8 warps take chunks in order from an atomic counter (chunk_rows():
+//     FOR / DFOR 16384 rows = 8 warps x 2 tiles x 2 sub-rounds, RFOR and the sizes pass 8192
+//     rows = 8 warps x 2 tiles); each warp loads its tiles (coalesced 16-byte loads) into
+//     shared memory;
 //   * the warp plans its tile: FOR blocks of 128 (ref = signed min, R4; per-miniblock
 //     bitwidth = bit length of the OR of the offsets, == bit length of the max, R3; neutral
 //     pads, R8), DFOR delta slots (R12, R13: slot s = x[s+1] - x[s], pads neutral), RFOR runs

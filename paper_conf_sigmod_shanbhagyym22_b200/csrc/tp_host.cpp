@@ -386,6 +386,23 @@ tp_status tp_shard(const tp_column* c, uint64_t row_lo, uint64_t row_hi, uint32_
   const uint64_t per = (rf || c->scheme == TP_NONE) ? kTile : kBlock;
   const uint64_t b0 = row_lo / per, b1 = (row_hi + per - 1) / per;
   *view = *c;
+  if (row_lo == row_hi) {  // an empty range (also of an empty column): no blocks, no words
+    view->n = 0;
+    view->num_blocks = 0;
+    r0[0] = 0;
+    memset(r0 + 1, 0, kGuard * 4);
+    view->starts0 = r0;
+    view->words0 = 0;
+    view->max_tile_words0 = 0;
+    if (rf) {
+      r1[0] = 0;
+      memset(r1 + 1, 0, kGuard * 4);
+      view->starts1 = r1;
+      view->words1 = 0;
+      view->max_tile_words1 = 0;
+    }
+    return TP_OK;
+  }
   view->n = row_hi - row_lo;
   view->num_blocks = b1 - b0;
   const bool dfor = c->scheme == TP_DFOR;
@@ -407,6 +424,94 @@ tp_status tp_shard(const tp_column* c, uint64_t row_lo, uint64_t row_hi, uint32_
     view->data1 = c->data1 + base1;
     view->words1 = c->starts1[b1] - base1;
   }
+  return TP_OK;
+}
+
+// Format check of a HOST column (include/tilepack.h tp_validate): header fields, block_starts
+// monotone and inside the data, every bitwidth byte <= 32 (R3, R5) and unused bytes zero,
+// every block exactly as long as its header says (Alg. 1 lines 13-14: 2 + sum of b words;
+// RFOR layout B, R17: 6 + tight miniblocks), RFOR run counts <= the block's rows; the exact
+// max_tile_words of each stream (what the decoders size their shared-memory ring with).
+tp_status tp_validate(const tp_column* c, uint32_t* mtw0_out, uint32_t* mtw1_out) {
+  if (!c) return TP_EINVAL;
+  const uint64_t n = c->n;
+  if (n >= (1ull << 32) || c->words0 >= (1ull << 32) || c->words1 >= (1ull << 32)) return TP_EUNSUPPORTED;
+  const uint32_t sch = c->scheme;
+  const bool rf = sch == TP_RFOR;
+  uint64_t per;
+  uint32_t mbc;
+  if (sch == TP_FOR || sch == TP_DFOR) { per = kBlock; mbc = 4; }
+  else if (sch == TP_FORNM) { per = kBlock; mbc = 1; }
+  else if (rf) { per = kTile; mbc = 16; }
+  else if (sch == TP_NONE) { per = kTile; mbc = 1; }
+  else return TP_EINVAL;
+  if (c->block_size != per || c->miniblock_count != mbc || c->num_blocks != (n + per - 1) / per) return TP_EFORMAT;
+  if (!c->starts0 || (c->words0 && !c->data0) || (rf && (!c->starts1 || (c->words1 && !c->data1))))
+    return TP_EINVAL;
+  const uint64_t nb = c->num_blocks;
+  const uint32_t* s0 = c->starts0;
+  uint32_t mtw0 = 0, mtw1 = 0;
+  for (uint64_t b = 0; b < nb; ++b)
+    if (s0[b] > s0[b + 1]) return TP_EFORMAT;
+  if (s0[nb] != c->words0) return TP_EFORMAT;
+  if (sch == TP_NONE) {
+    for (uint64_t b = 0; b < nb; ++b)
+      if (s0[b] != b * kTile) return TP_EFORMAT;
+    if (c->words0 < n) return TP_EFORMAT;
+    mtw0 = kTile;
+  } else if (!rf) {
+    const bool dfor = sch == TP_DFOR;
+    for (uint64_t b = 0; b < nb; ++b) {
+      // DFOR: the tile's first value precedes its first block (Fig. 6)
+      const uint64_t start = s0[b];
+      if (dfor && (b % 4) == 0 && start < 1) return TP_EFORMAT;
+      const uint64_t next = (dfor && (b + 1) % 4 == 0 && b + 1 < nb) ? (uint64_t)s0[b + 1] - 1 : s0[b + 1];
+      if (next < start + 2 || next > c->words0) return TP_EFORMAT;
+      const uint32_t bw = c->data0[start + 1];
+      uint32_t words = 2;
+      for (uint32_t j = 0; j < 4; ++j) {
+        const uint32_t bj = (bw >> (8 * j)) & 255u;
+        if (j >= mbc ? bj != 0 : bj > 32) return TP_EFORMAT;
+        words += mbc == 1 ? 4 * bj : bj;
+      }
+      if (next - start != words) return TP_EFORMAT;
+    }
+    for (uint64_t t = 0; 4 * t < nb; ++t) {
+      const uint64_t lo = dfor ? (uint64_t)s0[4 * t] - 1 : s0[4 * t];
+      const uint64_t hi = std::min<uint64_t>(4 * t + 4, nb) == nb ? c->words0
+                          : (dfor ? (uint64_t)s0[4 * t + 4] - 1 : s0[4 * t + 4]);
+      mtw0 = std::max<uint32_t>(mtw0, (uint32_t)(hi - lo));
+    }
+  } else {
+    const uint32_t* s1 = c->starts1;
+    for (uint64_t b = 0; b < nb; ++b)
+      if (s1[b] > s1[b + 1]) return TP_EFORMAT;
+    if (s1[nb] != c->words1) return TP_EFORMAT;
+    for (int q = 0; q < 2; ++q) {
+      const uint32_t* st = q ? s1 : s0;
+      const uint32_t* d = q ? c->data1 : c->data0;
+      uint32_t& mtw = q ? mtw1 : mtw0;
+      for (uint64_t b = 0; b < nb; ++b) {
+        const uint64_t start = st[b], span = (uint64_t)st[b + 1] - start;
+        if (span < 6) return TP_EFORMAT;
+        const uint32_t rows = (uint32_t)std::min<uint64_t>(kTile, n - b * kTile);
+        const uint32_t r = d[start];
+        if (r > rows || (rows > 0 && r == 0)) return TP_EFORMAT;
+        uint64_t words = 6;
+        for (uint32_t j = 0; j < 16; ++j) {
+          const uint32_t bj = (d[start + 2 + j / 4] >> (8 * (j % 4))) & 255u;
+          const uint32_t cnt = r > 32 * j ? std::min(32u, r - 32 * j) : 0u;
+          if (bj > 32 || (cnt == 0 && bj != 0)) return TP_EFORMAT;
+          words += (cnt * bj + 31) / 32;
+        }
+        if (span != words) return TP_EFORMAT;
+        if (q == 0 && d[start] != c->data1[s1[b]]) return TP_EFORMAT;  // both streams count the same runs
+        mtw = std::max<uint32_t>(mtw, (uint32_t)span);
+      }
+    }
+  }
+  if (mtw0_out) *mtw0_out = mtw0;
+  if (mtw1_out) *mtw1_out = mtw1;
   return TP_OK;
 }
 

@@ -94,7 +94,7 @@ __device__ __forceinline__ MbView fornm_mb(const Params& P, const Col& c, const 
     const uint32_t bs = v.ss[v.sshift + lb];
     const uint32_t* blk = v.sd + (bs - v.lo + v.dshift);
     m.ref = blk[0];
-    m.b = min(blk[1] & 255u, 32u);
+    m.b = checked_bw(blk[1] & 255u);
     m.w = blk + 2u + (g.mb & 3u) * m.b;
   } else {
     m.ref = 0u; m.b = 0u; m.w = v.sd;
@@ -206,7 +206,7 @@ __device__ __forceinline__ void rfor_scatter(const uint32_t* bV, const uint32_t*
   const uint32_t e0 = C * lane, m = e0 >> 5, pos = e0 & 31u;
   const uint32_t refV = bV[1], refL = bL[1];  // references (FOR on both arrays)
   const uint4 wv = make_uint4(bV[2], bV[3], bV[4], bV[5]), wl = make_uint4(bL[2], bL[3], bL[4], bL[5]);
-  const uint32_t bv = min(byte_of(wv, m), 32u), bl = min(byte_of(wl, m), 32u);  // R2, R17
+  const uint32_t bv = checked_bw(byte_of(wv, m)), bl = checked_bw(byte_of(wl, m));  // R2, R17
   // every miniblock before m is full: b_i words each (R17)
   const uint32_t* mV = bV + 6 + bytes_before(wv, m);
   const uint32_t* mL = bL + 6 + bytes_before(wl, m);
@@ -250,7 +250,11 @@ __device__ __forceinline__ void rfor_scatter_round(const Params& P, const Col& c
     if (C.t0s + tl >= C.tile_end) continue;  // warp-uniform; rows masked by the consumer
     const uint32_t* bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
     const uint32_t* bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
-    const uint32_t r = min(bV[0], 512u);  // run / value count
+    uint32_t r = bV[0];  // run / value count
+    if (r > 512u) {
+      tp_flag_error(4u);  // TP_DEVERR_RUNS
+      r = 512u;
+    }
     // C = entries per lane: the fewest that cover the block's runs (long runs: one entry per lane)
     if (SMALLC && r <= 32u) rfor_scatter<1>(bV, bL, r, lane, A, F);
     else if (SMALLC && r <= 64u) rfor_scatter<2>(bV, bL, r, lane, A, F);
@@ -455,6 +459,10 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
             const uintptr_t a1 = (reinterpret_cast<uintptr_t>(st.data + myhi) + 15) & ~uintptr_t(15);
             dsrc = reinterpret_cast<const char*>(a0);
             dbytes = (uint32_t)(a1 - a0);
+            if (dbytes > st.data_cap) {  // max_tile_words below the column's real span
+              tp_flag_error(2u);         // TP_DEVERR_TILE_WORDS: copy what fits, stay in the ring
+              dbytes = st.data_cap;
+            }
             const uint32_t s0 = st.kind == K_RFOR ? tile_base : 4u * tile_base;
             const uint32_t s1 = min(st.kind == K_RFOR ? tile_end : 4u * tile_end, st.nblocks) + 1u;
             const uintptr_t b0 = reinterpret_cast<uintptr_t>(st.starts + s0) & ~uintptr_t(15);
@@ -605,7 +613,7 @@ struct SumOp : OpBase {
         m = for_mb(P, c, C, g, sv, tl, tv);
         // a round whose TPR tiles are all inside the CTA range needs no row mask (CTA-uniform)
         const uint32_t tend = C.t0s + C.round_base + TPR;
-        const bool full_round = tend <= C.tile_end && tend * (uint32_t)TILE_ROWS <= P.n;
+        const bool full_round = tend <= C.tile_end && (uint64_t)tend * TILE_ROWS <= P.n;
         alive = full_round ? 0xffffffffu : valid_rows(P, C, g);
         full = full_round || __all_sync(FULL, alive == 0xffffffffu);
       } else {
@@ -991,7 +999,18 @@ struct StarOp : OpBase {
         if (A->mstage[c]) {
 #pragma unroll
           for (int i = 0; i < 32; ++i) W[32u * i + lane] = v[i];
-        } else if (!GROUPED) {
+        } else if (GROUPED) {
+          // only a DFOR aggregating measure gets here (others go sparse): its alive rows
+          uint32_t m = alive;
+          while (m) {
+            const uint32_t i = __ffs(m) - 1u;
+            m &= m - 1u;
+            int64_t y = (int32_t)v[i];
+            if (A->agg == TP_AGG_MUL) y *= (int64_t)(int32_t)W[32u * i + lane];
+            else if (A->agg == TP_AGG_SUB) y = (int64_t)(int32_t)W[32u * i + lane] - y;
+            ht_add(A->gzero ? 0u : G[32u * i + lane], y);
+          }
+        } else {
           const uint32_t m = alive;
           if (A->agg == TP_AGG_MUL) {
 #pragma unroll
@@ -1185,7 +1204,7 @@ __global__ void __launch_bounds__(256) k_bitmap_sum(const __grid_constant__ Para
         const uint32_t s = __ldg(st.starts + (mb >> 2));
         ref = __ldg(st.data + s);
         const uint32_t bw = __ldg(st.data + s + 1);
-        b = min((bw >> (8u * (mb & 3u))) & 255u, 32u);
+        b = checked_bw((bw >> (8u * (mb & 3u))) & 255u);
         mw = st.data + s + 2 + bw_prefix(bw, mb & 3u);
       }
       uint32_t e[32];
@@ -1203,7 +1222,7 @@ __global__ void __launch_bounds__(256) k_bitmap_sum(const __grid_constant__ Para
         first = __ldg(st.data + __ldg(st.starts + 4u * t) - 1u);
         ref = __ldg(st.data + s);
         const uint32_t bw = __ldg(st.data + s + 1);
-        b = min((bw >> (8u * (mb & 3u))) & 255u, 32u);
+        b = checked_bw((bw >> (8u * (mb & 3u))) & 255u);
         mw = st.data + s + 2 + bw_prefix(bw, mb & 3u);
       }
       uint32_t e[32];
@@ -1234,7 +1253,11 @@ __global__ void __launch_bounds__(256) k_bitmap_sum(const __grid_constant__ Para
         if (th >= P.ntiles || !((any >> (16u * h)) & 0xffffu)) continue;  // warp-uniform
         const uint32_t* bV = st.data + __ldg(st.starts + th);
         const uint32_t* bL = sl.data + __ldg(sl.starts + th);
-        const uint32_t r = min(__ldg(bV), 512u);
+        uint32_t r = __ldg(bV);
+        if (r > 512u) {
+          tp_flag_error(4u);  // TP_DEVERR_RUNS
+          r = 512u;
+        }
         if (r <= 32u) rfor_scatter<1>(bV, bL, r, lane, A, F);
         else if (r <= 64u) rfor_scatter<2>(bV, bL, r, lane, A, F);
         else if (r <= 128u) rfor_scatter<4>(bV, bL, r, lane, A, F);
@@ -1426,7 +1449,10 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
         continue;
       }
       st.data_off = off;
-      off += align4(std::max<uint32_t>(TPS * mtws[q] + 12u, 48u));  // + alignment slop + unpack over-read
+      const uint32_t region = align4(std::max<uint32_t>(TPS * mtws[q] + 12u, 48u));  // + alignment slop + unpack over-read
+      // bytes the producer may copy: the region minus the unpack over-read words (16-byte multiple)
+      st.data_cap = (region - 8u) * 4u & ~15u;
+      off += region;
       st.starts_off = off;
       off += align4((st.kind == K_RFOR ? TPS + 1u : 4u * TPS + 1u) + 8u);
     }
@@ -1733,6 +1759,17 @@ tp_status tp_bitmap_sum(const tp_column* dcol, const uint32_t* d_bitmap, int64_t
 }
 
 uint64_t tp_launch_count(void) { return g_launches.load(); }
+
+tp_status tp_device_errors(uint32_t* flags, void* stream) {
+  if (!flags) return TP_EINVAL;
+  if (cudaStreamSynchronize((cudaStream_t)stream) != cudaSuccess) return TP_ECUDA;
+  uint32_t v = 0;
+  if (cudaMemcpyFromSymbol(&v, g_tp_err, sizeof(v)) != cudaSuccess) return TP_ECUDA;
+  static const uint32_t zero = 0;
+  if (cudaMemcpyToSymbol(g_tp_err, &zero, sizeof(zero)) != cudaSuccess) return TP_ECUDA;
+  *flags = v;
+  return TP_OK;
+}
 
 /* profiling builds (-DTP_PROFILE_WAITS): copy out and reset the cycle counters */
 tp_status tp_debug_counters(uint64_t* out16) {

@@ -1,0 +1,103 @@
+// tp_roof.cu -- the measured INT32 issue roof ("Issue roof = measured INT32
+// throughput (bench microbenchmark of SHF/LOP3/IADD at 148 SMs)").  The low-bitwidth decoders
+// are bound by integer instruction issue, not by HBM (SURVEY finding 4, App. C.4; the paper's
+// DFOR is "bounded by shared memory bandwidth"), so their roofline denominator is
+// the rate at which the SMs retire the instructions the decode consists of: funnel shifts
+// (SHF), masks (LOP3), adds (IADD3) -- the ALU pipe -- and IMAD on the FMA pipe.
+//
+// One kernel, every SM full (8 CTAs x 256 threads), 8 independent dependency chains per thread
+// (enough ILP to cover the 4-cycle ALU latency), every operation inline PTX whose operands
+// change per iteration so ptxas can neither fold nor merge them (checked in the SASS: one SHF /
+// LOP3 / IADD3 / IMAD per PTX op).  kind: 0 SHF, 1 LOP3, 2 IADD3, 3 IMAD, 4 SHF+LOP3+IADD3 (the
+// unpack-and-sum mix of the decoders, all ALU pipe), 5 alternating LOP3 / IMAD (ALU + FMA pipes
+// dual-issued: the per-SMSP issue limit of one warp instruction per cycle).
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdint>
+
+#include "tilepack.h"
+
+namespace tp {
+extern std::atomic<uint64_t> g_launches;
+}
+
+namespace {
+
+constexpr int ROOF_THREADS = 256, ROOF_CTAS_PER_SM = 8, ROOF_CHAINS = 8, ROOF_UNROLL = 16;
+
+__device__ __forceinline__ uint32_t op_shf(uint32_t a, uint32_t b, uint32_t s) {
+  uint32_t d;
+  asm volatile("shf.r.wrap.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(s));
+  return d;
+}
+__device__ __forceinline__ uint32_t op_lop3(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t d;
+  asm volatile("lop3.b32 %0, %1, %2, %3, 0x96;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+  return d;
+}
+// three addends: one IADD3 (a two-operand add may be issued as IMAD on the FMA pipe)
+__device__ __forceinline__ uint32_t op_add(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t d;
+  asm volatile("{\n\t.reg .u32 t;\n\tadd.u32 t, %1, %2;\n\tadd.u32 %0, t, %3;\n\t}" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+  return d;
+}
+__device__ __forceinline__ uint32_t op_mad(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t d;
+  asm volatile("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+  return d;
+}
+
+template <int KIND>
+__global__ void __launch_bounds__(ROOF_THREADS) k_int_roof(uint32_t iters, uint32_t seed, uint32_t* sink) {
+  uint32_t a[ROOF_CHAINS];
+#pragma unroll
+  for (int c = 0; c < ROOF_CHAINS; ++c) a[c] = seed * (threadIdx.x + 1u) + (uint32_t)c * 0x9E3779B9u;
+  uint32_t k = seed ^ blockIdx.x;
+  for (uint32_t it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < ROOF_UNROLL; ++u) {
+#pragma unroll
+      for (int c = 0; c < ROOF_CHAINS; ++c) {
+        const uint32_t o = a[(c + 1) % ROOF_CHAINS];  // the previous value of a neighbour chain
+        if (KIND == 0) a[c] = op_shf(a[c], o, k);
+        else if (KIND == 1) a[c] = op_lop3(a[c], o, k);
+        else if (KIND == 2) a[c] = op_add(a[c], o, k);
+        else if (KIND == 3) a[c] = op_mad(a[c], o, k);
+        else if (KIND == 4) a[c] = (u % 3 == 0) ? op_shf(a[c], o, k) : (u % 3 == 1) ? op_lop3(a[c], o, k) : op_add(a[c], o, k);
+        else a[c] = (c & 1) ? op_mad(a[c], o, k) : op_lop3(a[c], o, k);
+      }
+    }
+    k += 0x61C88647u;
+  }
+  uint32_t r = 0;
+#pragma unroll
+  for (int c = 0; c < ROOF_CHAINS; ++c) r ^= a[c];
+  if (r == 0x12345678u) sink[0] = r;  // keeps the chains live; practically never stored
+}
+
+}  // namespace
+
+extern "C" {
+
+tp_status tp_bench_int_roof(int kind, uint32_t iters, uint32_t* d_sink, uint64_t* warp_insts, void* stream) {
+  if (kind < 0 || kind > 5 || !d_sink || !warp_insts || iters == 0) return TP_EINVAL;
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int grid = sms * ROOF_CTAS_PER_SM;
+  auto s = (cudaStream_t)stream;
+  switch (kind) {
+    case 0: k_int_roof<0><<<grid, ROOF_THREADS, 0, s>>>(iters, 12345u, d_sink); break;
+    case 1: k_int_roof<1><<<grid, ROOF_THREADS, 0, s>>>(iters, 12345u, d_sink); break;
+    case 2: k_int_roof<2><<<grid, ROOF_THREADS, 0, s>>>(iters, 12345u, d_sink); break;
+    case 3: k_int_roof<3><<<grid, ROOF_THREADS, 0, s>>>(iters, 12345u, d_sink); break;
+    case 4: k_int_roof<4><<<grid, ROOF_THREADS, 0, s>>>(iters, 12345u, d_sink); break;
+    default: k_int_roof<5><<<grid, ROOF_THREADS, 0, s>>>(iters, 12345u, d_sink); break;
+  }
+  tp::g_launches.fetch_add(1, std::memory_order_relaxed);
+  *warp_insts = (uint64_t)grid * (ROOF_THREADS / 32) * iters * ROOF_UNROLL * ROOF_CHAINS;
+  return cudaGetLastError() == cudaSuccess ? TP_OK : TP_ECUDA;
+}
+
+}  // extern "C"

@@ -76,6 +76,8 @@ def _load():
         "tp_choose_scheme": (i32, [vp, u64, vp, vp]),
         "tp_compressed_bytes": (u64, [colp]),
         "tp_shard": (i32, [colp, u64, u64, vp, vp, colp]),
+        "tp_validate": (i32, [colp, vp, vp]),
+        "tp_device_errors": (i32, [vp, vp]),
         "tp_decode": (i32, [colp, vp, vp]),
         "tp_decode_sum": (i32, [colp, vp, vp]),
         "tp_select_project_sum": (i32, [colp, i32, vp, vp, i32, i32, i32, vp, vp]),
@@ -92,6 +94,7 @@ def _load():
         "tp_gpu_encode_launch": (i32, [i32, vp, u64, vp, vp, u64, vp, vp, u64, vp, vp]),
         "tp_gpu_encode_result": (i32, [i32, u64, vp, vp, vp, vp, vp, colp, vp]),
         "tp_gpu_encode": (i32, [i32, vp, u64, vp, vp, u64, vp, vp, u64, vp, colp, vp]),
+        "tp_bench_int_roof": (i32, [i32, u32, vp, vp, vp]),
         "tp_status_string": (ctypes.c_char_p, [i32]),
         "tp_launch_count": (u64, []),
         "tp_debug_counters": (i32, [vp]),
@@ -162,6 +165,23 @@ def tp_shard(col: tp_column, row_lo: int, row_hi: int, rebased0, rebased1=None) 
     _check(_lib.tp_shard(ctypes.byref(col), row_lo, row_hi, _ptr(rebased0), _ptr(rebased1), ctypes.byref(view)),
            "tp_shard")
     return view
+
+
+def tp_validate(col: tp_column):
+    """Format check of a HOST column; returns (max_tile_words0, max_tile_words1)."""
+    m0, m1 = ctypes.c_uint32(), ctypes.c_uint32()
+    _check(_lib.tp_validate(ctypes.byref(col), ctypes.byref(m0), ctypes.byref(m1)), "tp_validate")
+    return m0.value, m1.value
+
+
+TP_DEVERR_BITWIDTH, TP_DEVERR_TILE_WORDS, TP_DEVERR_RUNS = 1, 2, 4
+
+
+def tp_device_errors(stream=None) -> int:
+    """Format-violation flags seen by the device calls since the last read (cleared); syncs."""
+    f = ctypes.c_uint32()
+    _check(_lib.tp_device_errors(ctypes.byref(f), _stream(stream)), "tp_device_errors")
+    return f.value
 
 
 def tp_decode(dcol: tp_column, d_out, stream=None):
@@ -281,6 +301,40 @@ def bitmap_sum(dcol, d_bitmap, out=None, stream=None):
 
 def tp_plain_sum(d_x, n: int, d_sum, stream=None):
     _check(_lib.tp_plain_sum(_ptr(d_x), n, _ptr(d_sum), _stream(stream)), "tp_plain_sum")
+
+
+def tp_bench_int_roof(kind: int, iters: int, d_sink, stream=None) -> int:
+    """Launch the INT32 issue-roof microbenchmark; returns the warp instructions it executes."""
+    w = ctypes.c_uint64()
+    _check(_lib.tp_bench_int_roof(kind, iters, _ptr(d_sink), ctypes.byref(w), _stream(stream)), "tp_bench_int_roof")
+    return w.value
+
+
+INT_ROOF_KINDS = {0: "SHF", 1: "LOP3", 2: "IADD3", 3: "IMAD", 4: "SHF+LOP3+IADD3 (ALU pipe)",
+                  5: "LOP3+IMAD (ALU+FMA pipes)"}
+
+
+def measure_int_roof(iters: int = 4000, reps: int = 5, stream=None) -> dict:
+    """The measured INT32 issue roof: warp instructions / s over all SMs per
+    kind, best of `reps` CUDA-event-timed launches after a warm-up."""
+    import torch
+    sink = torch.zeros(1, dtype=torch.int32, device="cuda")
+    s = stream if stream is not None else torch.cuda.current_stream()
+    out = {}
+    for kind, name in INT_ROOF_KINDS.items():
+        tp_bench_int_roof(kind, 64, sink, s)
+        best = None
+        for _ in range(reps):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(s)
+            w = tp_bench_int_roof(kind, iters, sink, s)
+            b.record(s)
+            torch.cuda.synchronize()
+            ms = a.elapsed_time(b)
+            best = ms if best is None or ms < best else best
+        out[name] = {"warp_insts": w, "ms": best, "warp_insts_per_s": w / (best / 1e3),
+                     "lane_ops_per_s": 32 * w / (best / 1e3)}
+    return out
 
 
 def tp_debug_counters():

@@ -125,6 +125,61 @@ def test_bench_size_for_b16_sampled():
     assert np.array_equal(got, x[idx])
     tail = out[n - 1000:].cpu().numpy()
     assert np.array_equal(tail, oracle.for_decode_range(e, n - 1000, n, dg))
+    # the whole decoded column == x (decode(encode(x)) == x, the oracle-pinned definition)
+    assert torch.equal(out, torch.from_numpy(x).cuda())
+    assert tp.tp_device_errors() == 0
+
+
+@pytest.mark.parametrize("b", [0, 1, 4, 8, 12])
+def test_lean_for_sum_full_rounds(b):
+    """The low-bitwidth decode->sum variant (k_decode_sum<FOR, LEAN>, max_tile_words <= 200) on a
+    column long enough that every CTA runs many full rounds of 8 tiles per item (24M rows = 46,875
+    tiles over <= 740 CTAs), plus a ragged tail: the fused sum == the int64 sum of x, the decoded
+    column == x element by element (Alg. 1; bitwidth sweep P:1419-1423)."""
+    n = 24_000_000 + 333
+    x = datagen.uniform_bits(b, n, seed=7000 + b)
+    h = tp.encode(x, "for")
+    assert h.col.max_tile_words0 <= 200  # the lean kernel is the one dispatched
+    d = h.to_device()
+    assert int(tp.decode_sum(d).item()) == oracle.column_sum(x)
+    xd = torch.from_numpy(x).cuda()
+    assert torch.equal(tp.decode(d), xd)
+    # every 512-row tile-range shard boundary inside a CTA's range: a sub-range starting mid-column
+    from paper_conf_sigmod_shanbhagyym22_b200 import dist as tpd
+    lo, hi = tpd.tile_range(n, 1, 3)
+    ds = tpd.ShardColumn(h, lo, hi).to_device()
+    assert int(tp.decode_sum(ds).item()) == oracle.column_sum(x[lo:hi])
+    assert tp.tp_device_errors() == 0
+
+
+def test_device_format_errors_flagged():
+    """Format violations the kernels meet are flagged (tp_device_errors), not silent: a bitwidth
+    byte > 32 (R3, R5) and a max_tile_words below the column's real tile span (the ring stays in
+    bounds, the flag says the result is undefined)."""
+    assert tp.tp_device_errors() == 0
+    x = datagen.uniform_bits(10, 512 * 64 + 5, seed=3)
+    h = tp.encode(x, "for")
+    d = h.to_device()
+    tp.decode_sum(d)
+    assert tp.tp_device_errors() == 0
+    bw = int(h.starts0[9]) + 1
+    bad = h.data0.copy()
+    bad[bw] = (bad[bw] & ~np.uint32(0xff0000)) | np.uint32(45 << 16)
+    d.data0.copy_(torch.from_numpy(bad.view(np.int32)))
+    tp.decode_sum(d)
+    assert tp.tp_device_errors() & tp.TP_DEVERR_BITWIDTH
+    d = h.to_device()
+    d.col.max_tile_words0 = 8  # far below the 4 x (2 + 4 x 10) words of a tile
+    tp.decode_sum(d)
+    assert tp.tp_device_errors() & tp.TP_DEVERR_TILE_WORDS
+    r = tp.encode(datagen.runs(512 * 8, 4, seed=2), "rfor")
+    dr = r.to_device()
+    bad = r.data0.copy()
+    bad[int(r.starts0[3])] = 900  # run count > 512
+    dr.data0.copy_(torch.from_numpy(bad.view(np.int32)))
+    tp.decode_sum(dr)
+    assert tp.tp_device_errors() & tp.TP_DEVERR_RUNS
+    assert tp.tp_device_errors() == 0  # read-and-clear
 
 
 @pytest.mark.parametrize("scheme", SCHEMES)

@@ -141,3 +141,60 @@ def test_gpu_encode_bound_covers_every_encoding():
     x = datagen.uniform_bits(32, 128 * 40, seed=4)
     assert tp.tp_gpu_encode_bound(tp.TP_FOR, len(x))[1] == tp.encode(x, "for").col.words0
     assert tp.tp_gpu_encode_workspace_bytes(10**8) > tp.tp_gpu_encode_workspace_bytes(10**6) > 0
+
+
+@pytest.mark.parametrize("scheme", ("for", "dfor", "rfor", "none", "fornm"))
+def test_validate_accepts_encoder_output(scheme):
+    """tp_validate accepts every encoded column and reports the encoder's max_tile_words."""
+    for name, x in list(datagen.mixed_columns(seed=8)) + [("c16", datagen.uniform_bits(16, 100_003, seed=1))]:
+        h = tp.encode(x, scheme)
+        m0, m1 = tp.tp_validate(h.col)
+        assert (m0, m1) == (h.col.max_tile_words0, h.col.max_tile_words1), (scheme, name)
+
+
+def _expect_eformat(col):
+    with pytest.raises(tp.TilepackError, match="malformed"):
+        tp.tp_validate(col)
+
+
+def test_validate_rejects_corruptions():
+    """Each corruption a decoder could not survive is TP_EFORMAT (include/tilepack.h tp_validate)."""
+    x = datagen.uniform_bits(9, 512 * 6 + 40, seed=2)
+    h = tp.encode(x, "for")
+    bw_word = int(h.starts0[3]) + 1
+    old = h.data0[bw_word]
+    h.data0[bw_word] = (old & ~np.uint32(0xff00)) | np.uint32(40 << 8)   # bitwidth byte 40 > 32
+    _expect_eformat(h.col)
+    h.data0[bw_word] = old
+    tp.tp_validate(h.col)
+    h.starts0[5], h.starts0[6] = h.starts0[6], h.starts0[5]              # block_starts not monotone
+    _expect_eformat(h.col)
+    h = tp.encode(x, "for")
+    h.col.num_blocks = h.col.num_blocks - 1                               # header inconsistent with n
+    _expect_eformat(h.col)
+    h = tp.encode(x, "fornm")
+    h.data0[int(h.starts0[2]) + 1] |= np.uint32(1 << 8)                   # FORNM: bytes 1..3 must be 0
+    _expect_eformat(h.col)
+    r = tp.encode(datagen.runs(512 * 4, 5, seed=1), "rfor")
+    r.data0[int(r.starts0[1])] = 600                                      # run count > 512
+    _expect_eformat(r.col)
+    r = tp.encode(datagen.runs(512 * 4, 5, seed=1), "rfor")
+    r.data1[int(r.starts1[2])] += 1                                       # streams disagree on the run count
+    _expect_eformat(r.col)
+    d = tp.encode(datagen.near_sorted(512 * 3 + 9, seed=3), "dfor")
+    d.col.words0 = d.col.words0 - 1                                       # data shorter than block_starts says
+    _expect_eformat(d.col)
+
+
+@pytest.mark.parametrize("scheme", ("for", "dfor", "rfor", "none"))
+def test_shard_empty_range(scheme):
+    """An empty tile range (and a shard of an empty column) is an empty view, no underflow."""
+    from paper_conf_sigmod_shanbhagyym22_b200 import dist as tpd
+    x = datagen.uniform_bits(5, 512 * 3, seed=1)
+    for col in (x, np.zeros(0, np.int32)):
+        h = tp.encode(col, scheme)
+        s = tpd.ShardColumn(h, 0, 0)
+        assert s.n == 0 and int(s.col.num_blocks) == 0 and int(s.col.words0) == 0 and int(s.col.words1) == 0
+    h = tp.encode(np.zeros(0, np.int32), scheme)
+    s = tpd.shard(h, 1, 4)
+    assert s.n == 0 and int(s.col.words0) == 0

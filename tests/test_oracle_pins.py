@@ -234,3 +234,42 @@ def test_bitmap_sum_pins():
     bm = datagen.bernoulli_bitmap(n, 0.01, seed=4)
     frac = np.unpackbits(bm.view(np.uint8), bitorder="little")[:n].mean()
     assert 0.005 < frac < 0.02
+
+
+def test_choose_scheme_tie_break_r20():
+    """R20 (P:1206-1208 silent on ties): equal footprints resolve FOR < DFOR < RFOR.  An empty
+    column encodes to the 3-word header + one block_starts entry under FOR and DFOR (16 B each)
+    and under RFOR to the header + two block_starts entries (20 B): FOR and DFOR tie -> FOR.
+    A single value: FOR 1 block [ref][bw] (+2 starts), DFOR 1 tile [first][0][0] (+2 starts):
+    FOR is strictly smaller, so the pin below is the tie itself, not an accident of sizes."""
+    x = np.zeros(0, np.int32)
+    sizes = {s: oracle.encode(s, x).nbytes() for s in ("for", "dfor", "rfor")}
+    assert sizes["for"] == sizes["dfor"] == 16 and sizes["rfor"] == 20
+    assert oracle.choose_scheme(x)[0] == "for"
+    # no tie: a constant tile is smallest under FOR (4 x [ref][0]) < DFOR (+ first) < RFOR (2 streams)
+    y = np.full(512, 7, np.int32)
+    s = {k: oracle.encode(k, y).nbytes() for k in ("for", "dfor", "rfor")}
+    assert s["for"] < s["dfor"] < s["rfor"]
+    assert oracle.choose_scheme(y)[0] == "for"
+
+
+def test_fornm_roundtrip_is_identity():
+    """GPU-FOR without miniblocks (one bitwidth per 128-value block) is lossless:
+    decode(encode(x)) == x, on ragged lengths, b = 0 / 32 and a skewed column; its size is
+    the closed form 4 (3 + nb + 1 + sum_blocks (2 + 4 b_block)) with b_block = bit length of
+    the block's max offset (R3 over the whole block)."""
+    for name, x in datagen.mixed_columns(seed=41):
+        e = oracle.encode("fornm", x)
+        assert np.array_equal(oracle.decode(e), x), name
+    rng = np.random.default_rng(6)
+    for x in (np.zeros(1000, np.int32), datagen.uniform_bits(32, 777, seed=2),
+              rng.integers(0, 2**5, 128 * 9 + 3, dtype=np.int64).astype(np.int32)):
+        e = oracle.encode("fornm", x)
+        assert np.array_equal(oracle.decode(e), x)
+        nb = -(-len(x) // 128)
+        words = 0
+        for k in range(nb):
+            blk = x[128 * k: 128 * k + 128].astype(np.int64)
+            off = int((blk - blk.min()).max())
+            words += 2 + 4 * off.bit_length()
+        assert e.nbytes() == 4 * (3 + nb + 1 + words)

@@ -136,3 +136,36 @@ def test_gpu_star_queries_sharded_sum_equals_whole():
             pp = e.prepare(qid)
             e.execute(pp, acc_s, acc_c)
         assert torch.equal(acc_s, sw) and torch.equal(acc_c, cw), qid
+
+
+def test_generator_rank_slices_concatenate():
+    """Rank-local generation (bench / multi-GPU): the row slices of the chunked generator are the
+    rows of the whole table, for ragged 512-row tile-range cuts."""
+    from paper_conf_sigmod_shanbhagyym22_b200.dist import tile_range
+    whole = gen.generate(0.3, seed=9)
+    n = whole["lineorder_rows"]
+    assert n == len(whole["lineorder"]["lo_orderdate"]) == gen.num_rows(0.3, seed=9)
+    for world in (3, 8):
+        parts = [gen.generate(0.3, seed=9, rows=tile_range(n, r, world)) for r in range(world)]
+        for c in ("lo_orderdate", "lo_custkey", "lo_revenue", "lo_supplycost"):
+            assert np.array_equal(np.concatenate([p["lineorder"][c] for p in parts]), whole["lineorder"][c])
+
+
+@pytest.mark.gpu
+@pytest.mark.slow
+def test_gpu_star_queries_sf20_match_golden():
+    """BASELINE config 5 at the bench's size (SF 20, 120M rows, GPU-* columns, the bench's launch
+    configuration): every query == the oracle's answer stored by scripts/make_ssb_golden.py
+    (oracle/ssb.py over the uncompressed columns)."""
+    import json
+    import os
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sigmod_shanbhagyym22_b200.ssb import SSBEngine
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "ssb_sf20.json")))
+    db = gen.generate(20, seed=g["seed"], columns=gen.QUERY_COLUMNS)
+    assert db["lineorder_rows"] == g["rows"]
+    eng = SSBEngine(db)
+    for qid in QUERIES:
+        assert [list(r) for r in eng.run(qid)] == g["results"][qid], qid
