@@ -77,10 +77,11 @@ def dist_env():
 
 # ------------------------------------------------------------------ clocks (NVML, during the timed region)
 class ClockSampler:
-    """Samples the SM clock and the clock-event reasons back to back (no sleep: an NVML query
-    takes ~0.1 ms, so even a few-ms timed region yields tens of samples)."""
+    """Samples the SM clock and the clock-event reasons every 0.5 ms (a sampler without a sleep
+    holds the GIL so often that the launching thread falls behind the GPU: measured 3.6x on a
+    20-step region)."""
 
-    def __init__(self, index: int, period: float = 0.0):
+    def __init__(self, index: int, period: float = 0.0005):
         self.samples, self.reasons, self.max_mhz = [], set(), None
         self.period, self._stop = period, threading.Event()
         try:
@@ -124,7 +125,7 @@ class ClockSampler:
     def summary(self):
         return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
                 "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples),
-                "source": "NVML (same counters as nvidia-smi), sampled back to back during the timed steps"}
+                "source": "NVML (same counters as nvidia-smi), sampled every 0.5 ms during the timed steps"}
 
 
 def measured_peak():

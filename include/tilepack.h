@@ -320,9 +320,10 @@ tp_status tp_gpu_encode(int scheme, const int32_t* d_x, uint64_t n, uint32_t* d_
  * Launches one microbenchmark kernel on every SM (8 CTAs x 256 threads, 8 independent
  * dependency chains per thread) asynchronously on `stream`; *warp_insts (host) = the
  * warp instructions of the measured kind it executes (the caller times the launch).
- * kind: 0 SHF, 1 LOP3, 2 IADD3, 3 IMAD, 4 SHF / LOP3 / IADD3 mix (ALU pipe only: the
- * unpack-and-sum mix), 5 LOP3 / IMAD alternating (ALU + FMA pipes: the per-SMSP issue
- * limit).  d_sink: one DEVICE u32 (practically never written). */
+ * kind (three register operands): 0 SHF, 1 LOP3, 2 IADD3, 3 IMAD, 4 SHF / LOP3 / IADD3
+ * mix (ALU pipe), 5 LOP3 / IMAD alternating (ALU + FMA pipes); (two registers + an
+ * immediate): 6 SHF, 7 LOP3, 8 IMAD, 9 LOP3 / SHF / IMAD over both pipes (the per-SMSP
+ * issue limit).  d_sink: one DEVICE u32 (practically never written). */
 tp_status tp_bench_int_roof(int kind, uint32_t iters, uint32_t* d_sink, uint64_t* warp_insts, void* stream);
 
 /* --------------------------------------------------------------- utility */

@@ -140,14 +140,12 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 // (include/tilepack.h tp_device_errors; one copy per translation unit -- the pipeline
 // kernels' copy in tp_kernels.cu is the one the ABI reads)
 static __device__ uint32_t g_tp_err;
-static __device__ __noinline__ void tp_flag_error(uint32_t bit) { atomicOr(&g_tp_err, bit); }
-// a miniblock bitwidth byte: > 32 is a format violation (R3, R5), used as 32
+__device__ __forceinline__ void tp_flag_error(uint32_t bit) { atomicOr(&g_tp_err, bit); }
+// a miniblock bitwidth byte: > 32 is a format violation (R3, R5), used as 32 (a predicated
+// RED on the rare path; no branch around the decode)
 __device__ __forceinline__ uint32_t checked_bw(uint32_t b) {
-  if (b > 32u) {
-    tp_flag_error(1u);  // TP_DEVERR_BITWIDTH
-    b = 32u;
-  }
-  return b;
+  if (__builtin_expect(b > 32u, 0)) tp_flag_error(1u);  // TP_DEVERR_BITWIDTH
+  return min(b, 32u);
 }
 
 // ------------------------------------------------------------------ column params
@@ -182,6 +180,7 @@ struct alignas(64) Params {
   uint32_t rounds;      // consumer rounds per item: an item holds TPR * rounds tiles of one column
   uint32_t agg_off;     // word offset of the per-CTA aggregation table
   uint32_t bar_off;     // word offset of the mbarriers (8-byte aligned)
+  uint32_t ring_words;  // query pipeline: words of the byte ring (at smem offset 0)
 };
 
 // ------------------------------------------------------------------ bit unpack

@@ -32,6 +32,7 @@ struct StageCtx {
   uint32_t t0s;           // first tile of the stage (global index)
   uint32_t round_base;    // stage-local index of the round's first tile
   uint32_t tile_end;      // one past the last tile of the CTA range
+  uint32_t doff[2], soff[2];  // word offsets of the item's data / block_starts regions per stream
 };
 
 struct StreamView {
@@ -43,12 +44,13 @@ struct StreamView {
 
 // Every lane derives the view itself (two smem loads + address arithmetic): cheaper on
 // the per-round critical path than sharing it through shared memory and a warp sync.
-__device__ __forceinline__ StreamView stream_view(const Params& P, uint32_t s, const StageCtx& C) {
+// s = the stream (Params::st index), k = 0 / 1: the column's first / second stream
+__device__ __forceinline__ StreamView stream_view(const Params& P, uint32_t s, const StageCtx& C, uint32_t k = 0) {
   const Stream& st = P.st[s];
   StreamView v;  // FOR / DFOR / RFOR streams only (a None column is read through none_row)
   const uint32_t sidx = st.kind == K_RFOR ? C.t0s : 4u * C.t0s;
-  v.ss = C.stage + st.starts_off;
-  v.sd = C.stage + st.data_off;
+  v.ss = C.stage + C.soff[k];
+  v.sd = C.stage + C.doff[k];
   v.sshift = align_shift(st.starts, sidx);
   v.lo = v.ss[v.sshift] - (st.kind == K_DFOR ? 1u : 0u);
   v.dshift = align_shift(st.data, v.lo);
@@ -237,7 +239,7 @@ __device__ __forceinline__ void rfor_scatter(const uint32_t* bV, const uint32_t*
 template <bool SMALLC = false>
 __device__ __forceinline__ void rfor_scatter_round(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                                    uint32_t* scratch) {
-  const StreamView vv = stream_view(P, c.s0, C), vl = stream_view(P, c.s1, C);
+  const StreamView vv = stream_view(P, c.s0, C, 0), vl = stream_view(P, c.s1, C, 1);
   const uint32_t lane = g.lane;
   __syncwarp();  // a lagging lane may still read the previous column's expansion
 #pragma unroll 1
@@ -334,7 +336,7 @@ __device__ __forceinline__ const uint32_t* none_row(const Params& P, const Col& 
                                                     const Lane& g, uint32_t& sw) {
   const uint32_t r = 16u * (C.round_base + g.tile_local) + g.mb;
   sw = r & 7u;
-  return C.stage + P.st[c.s0].data_off + 32u * r;
+  return C.stage + C.doff[0] + 32u * r;
 }
 __device__ __forceinline__ void decode_none(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                             uint32_t (&val)[32]) {
@@ -501,6 +503,12 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
         C.t0s = t0 + gi * TPS;
         C.stage = smem + slot * P.stage_words;
         const uint32_t nr = min(P.rounds, (t1 - C.t0s + TPR - 1) / TPR);
+        {
+          const Col& c0 = P.col[0];
+          C.doff[0] = P.st[c0.s0].data_off; C.soff[0] = P.st[c0.s0].starts_off;
+          const uint32_t q1 = c0.scheme == S_RFOR ? c0.s1 : c0.s0;
+          C.doff[1] = P.st[q1].data_off; C.soff[1] = P.st[q1].starts_off;
+        }
         if (Op::kProducerSpin) mbar_wait(&full[slot], phase); else mbar_wait_backoff(&full[slot], phase);
         for (uint32_t r = 0; r < nr; ++r, ++rc) {
           C.round_base = r * TPR;
@@ -520,6 +528,12 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
         op.begin(P, C, g);
         for (uint32_t c = 0; c < P.ncols; ++c) {
           C.stage = smem + slot * P.stage_words;
+          {
+            const Col& cc = P.col[c];
+            C.doff[0] = P.st[cc.s0].data_off; C.soff[0] = P.st[cc.s0].starts_off;
+            const uint32_t q1 = cc.scheme == S_RFOR ? cc.s1 : cc.s0;
+            C.doff[1] = P.st[q1].data_off; C.soff[1] = P.st[q1].starts_off;
+          }
 #ifdef TP_PROFILE_WAITS
           const long long w0 = clock64();
 #endif
@@ -539,6 +553,171 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
           if (++slot == P.nstages) { slot = 0; phase ^= 1u; }
         }
         op.end(P, C, g);
+      }
+    }
+    op.finish(P, g, smem);
+  }
+}
+
+// ------------------------------------------------------------------ the query pipeline
+// Multi-column operators (select / project / aggregate, star queries) stream one item per column
+// of each range of TPR tiles, in evaluation order.  The items of one query differ in size by up
+// to 10x (a 5.7-bit RFOR date column next to a 24-bit FOR price), so the ring is a BYTE ring:
+// the producer places each item at the next free 16-byte aligned offset (wrapping to the ring
+// start when it does not fit at the end; a None box 1024-byte aligned) and reclaims space as the
+// consumers release items, oldest first.  QNS item slots carry each item's mbarriers and layout
+// {ring offset, block_starts offset of stream 0, data / block_starts offsets of stream 1}.
+// The bytes in flight are the ring's whatever the column mix (fixed slots sized for the widest
+// column held two items of an SSB query).  An operator may keep an item (Op::col returns false:
+// the staged first measure, read back when the last column aggregates); it is released at the
+// end of its round -- the host sizes the ring so that the items in between always fit.
+constexpr uint32_t QNS = 16;
+
+template <class Op>
+__device__ __forceinline__ void run_query_pipeline(const Params& P, Op& op) {
+  extern __shared__ __align__(1024) uint32_t smem[];
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
+  const uint32_t npairs = (P.ntiles + 1u) >> 1;
+  const uint32_t p0 = (uint32_t)((uint64_t)blockIdx.x * npairs / gridDim.x);
+  const uint32_t p1 = (uint32_t)((uint64_t)(blockIdx.x + 1) * npairs / gridDim.x);
+  const uint32_t t0 = 2u * p0, t1 = min(2u * p1, P.ntiles);
+  if (t0 >= t1) return;
+  const uint32_t ngr = (t1 - t0 + TPR - 1) / TPR;
+  const uint32_t RW = P.ring_words;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + P.bar_off);
+  uint64_t* empty = full + QNS;
+  uint32_t* meta = reinterpret_cast<uint32_t*>(empty + QNS);  // 4 words per slot
+  op.cta_init(P, smem);
+  if (threadIdx.x == 0) {
+    for (uint32_t s = 0; s < QNS; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], CONSUMER_WARPS);
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+
+  if (warp == 0) {
+    // ---------------- producer
+    const uint64_t pol = policy_evict_first();
+    uint32_t head = 0;    // virtual word offset of the next allocation (monotonic)
+    uint32_t oldest = 0;  // the oldest item not yet seen released
+    uint32_t vst = 0;     // lane s < QNS: virtual start of the item in slot s
+    uint32_t item = 0;
+    for (uint32_t gb = 0; gb < ngr; gb += 31) {
+      const uint32_t tb = min(t0 + (gb + lane) * TPR, t1);
+      uint32_t bnd[MAX_STREAMS];
+#pragma unroll
+      for (int q = 0; q < MAX_STREAMS; ++q) {
+        bnd[q] = 0u;
+        if ((uint32_t)q < P.nstreams) {
+          const Stream& st = P.st[q];
+          bnd[q] = __ldg(st.starts + min(st.kind == K_RFOR ? tb : 4u * tb, st.nblocks));
+        }
+      }
+      const uint32_t ge = min(gb + 31, ngr);
+      for (uint32_t g = gb; g < ge; ++g) {
+        const uint32_t tile_base = t0 + g * TPR, tile_end = min(tile_base + TPR, t1);
+        for (uint32_t c = 0; c < P.ncols; ++c, ++item) {
+          const Col& cc = P.col[c];
+          const uint32_t my_s = lane == 0 ? cc.s0 : (lane == 1 && cc.scheme == S_RFOR ? cc.s1 : 0xffu);
+          uint32_t mylo = 0u, myhi = 0u;
+#pragma unroll
+          for (int q = 0; q < MAX_STREAMS; ++q) {
+            if ((uint32_t)q < P.nstreams) {
+              const uint32_t a = __shfl_sync(FULL, bnd[q], g - gb);
+              const uint32_t b = __shfl_sync(FULL, bnd[q], g - gb + 1);
+              if (my_s == (uint32_t)q) { mylo = a; myhi = b; }
+            }
+          }
+          const bool none = (Op::kMask & M_NONE) && cc.scheme == S_NONE;  // column-uniform
+          uint32_t dbytes = 0u, sbytes = 0u, dwords = 0u, swords = 0u;
+          const char *dsrc = nullptr, *ssrc = nullptr;
+          if (none) {
+            dwords = lane == 0 ? TPR * TILE_ROWS : 0u;  // one TMA tensor box (OOB rows zero-filled)
+            dbytes = 4u * dwords;
+          } else if (my_s != 0xffu) {
+            const Stream& st = P.st[my_s];
+            const uint32_t lo = mylo - (st.kind == K_DFOR ? 1u : 0u);
+            const uintptr_t a0 = reinterpret_cast<uintptr_t>(st.data + lo) & ~uintptr_t(15);
+            const uintptr_t a1 = (reinterpret_cast<uintptr_t>(st.data + myhi) + 15) & ~uintptr_t(15);
+            dsrc = reinterpret_cast<const char*>(a0);
+            dbytes = (uint32_t)(a1 - a0);
+            const uint32_t s0 = st.kind == K_RFOR ? tile_base : 4u * tile_base;
+            const uint32_t s1 = min(st.kind == K_RFOR ? tile_end : 4u * tile_end, st.nblocks) + 1u;
+            const uintptr_t b0 = reinterpret_cast<uintptr_t>(st.starts + s0) & ~uintptr_t(15);
+            const uintptr_t b1 = (reinterpret_cast<uintptr_t>(st.starts + s1) + 15) & ~uintptr_t(15);
+            ssrc = reinterpret_cast<const char*>(b0);
+            sbytes = (uint32_t)(b1 - b0);
+            swords = sbytes >> 2;
+            // a malformed column (a tile longer than max_tile_words says) must not outgrow the ring
+            const uint32_t cap = 4u * ((RW >> 1) - swords - 8u);
+            if (dbytes > cap) {
+              tp_flag_error(2u);  // TP_DEVERR_TILE_WORDS
+              dbytes = cap & ~15u;
+            }
+            dwords = (dbytes >> 2) + 4u;  // + the unpack's over-read (Alg. 1 line 15 reads word k + 1)
+          }
+          const uint32_t rw0 = __shfl_sync(FULL, dwords + swords, 0);
+          const uint32_t rw1 = __shfl_sync(FULL, dwords + swords, 1);
+          const uint32_t need = rw0 + rw1;  // multiples of 4 words
+          uint32_t hd = none ? (head + 255u) & ~255u : head;
+          if (hd % RW + need > RW) hd += RW - hd % RW;  // does not fit before the ring's end: wrap
+          // reclaim: the slot's previous item, and every item still holding the space needed
+          while (item - oldest >= QNS || (oldest < item && hd + need > __shfl_sync(FULL, vst, oldest % QNS) + RW)) {
+            mbar_wait_backoff(&empty[oldest % QNS], (oldest / QNS) & 1u);
+            ++oldest;
+          }
+          const uint32_t slot = item % QNS;
+          if (lane == slot) vst = hd;
+          head = hd + need;
+          const uint32_t off = hd % RW;
+          const uint32_t dw0 = __shfl_sync(FULL, dwords, 0), dw1 = __shfl_sync(FULL, dwords, 1);
+          if (lane == 0)  // stream 0: data at 0, block_starts at dw0; stream 1: data at rw0, starts after it
+            *reinterpret_cast<uint4*>(meta + 4u * slot) = make_uint4(off, dw0, rw0, rw0 + dw1);
+          const uint32_t total = __reduce_add_sync(FULL, dbytes + sbytes);
+          if (lane == 0) mbar_arrive_expect_tx(&full[slot], total);
+          __syncwarp();
+          uint32_t* dst = smem + off + (lane == 1 ? rw0 : 0u);
+          if (none) {
+            if (lane == 0) tma_load_2d(dst, &P.tmap[c], 0, (int)(tile_base * (TILE_ROWS / 32)), &full[slot], pol);
+          } else if (my_s != 0xffu) {
+            bulk_g2s(dst, dsrc, dbytes, &full[slot], pol);
+            bulk_g2s(dst + dwords, ssrc, sbytes, &full[slot], pol);
+          }
+        }
+      }
+    }
+  } else {
+    // ---------------- consumers
+    const Lane g = lane_geom();
+    uint32_t* scratch = smem + P.scratch_off + g.cw * P.scratch_words_per_warp;
+    uint32_t item = 0;
+    StageCtx C;
+    C.tile_end = t1;
+    C.round_base = 0;
+    for (uint32_t gi = 0; gi < ngr; ++gi) {
+      C.t0s = t0 + gi * TPR;
+      op.begin(P, C, g);
+      uint32_t held = 0xffffffffu;
+      for (uint32_t c = 0; c < P.ncols; ++c, ++item) {
+        const uint32_t slot = item % QNS;
+        mbar_wait_backoff(&full[slot], (item / QNS) & 1u);
+        const uint4 mt = *reinterpret_cast<const uint4*>(meta + 4u * slot);
+        C.stage = smem + mt.x;
+        C.doff[0] = 0u; C.soff[0] = mt.y; C.doff[1] = mt.z; C.soff[1] = mt.w;
+        const bool rel = op.col(P, C, g, scratch, c, gi);
+        __syncwarp();
+        if (rel) {
+          if (g.lane == 0) mbar_arrive(&empty[slot]);
+        } else {
+          held = slot;
+        }
+      }
+      op.end(P, C, g);
+      if (held != 0xffffffffu) {
+        __syncwarp();
+        if (g.lane == 0) mbar_arrive(&empty[held]);
       }
     }
     op.finish(P, g, smem);
@@ -731,8 +910,8 @@ struct SelectOp : OpBase {
   uint32_t alive;
   uint32_t va[32];
   __device__ void begin(const Params& P, const StageCtx& C, const Lane& g) { alive = valid_rows(P, C, g); }
-  __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c, uint32_t) {
-    if (!__any_sync(FULL, alive != 0u)) return;  // nothing survives in this warp's rows
+  __device__ bool col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c, uint32_t) {
+    if (!__any_sync(FULL, alive != 0u)) return true;  // nothing survives in this warp's rows
     uint32_t v[32];
     decode_col<MASK, TP_QUERY_COMPACT>(P, c, C, g, scratch, v);
     const int32_t l = A->lo[c], h = A->hi[c];
@@ -758,6 +937,7 @@ struct SelectOp : OpBase {
         }
       }
     }
+    return true;
   }
   __device__ void end(const Params&, const StageCtx&, const Lane&) {
     if (A->proj == TP_PROJ_COUNT) acc += __popc(alive);
@@ -772,30 +952,39 @@ struct SelectOp : OpBase {
 // SSB as one tile kernel: FK columns probe dimension lookup tables
 // (Crystal's perfect hash, key - key_min), payloads build a dense group index,
 // measures are aggregated per group.  Columns come in the host's order (most selective
-// first); the last column is the aggregating measure, a first measure (MUL / SUB) is staged.
+// first); the last column is the aggregating measure, a first measure (MUL / SUB) is read
+// back when it aggregates.
 //
-// Per column, a warp picks one of two evaluation modes (warp-uniform):
+// GPU-FOR / GPU-DFOR / None columns: per column a warp picks one of two evaluation modes
+// (warp-uniform):
 //  * dense  -- while many of its 1024 rows are alive: decode all 32 rows per thread
 //    (tile decode) and apply the column's role to each;
 //  * sparse -- once few rows survive: visit only the alive rows and read each one's value
 //    straight out of the staged tile (random access into a FOR miniblock, Alg. 1 for one
-//    entry; for RFOR, the run whose start precedes the row) -- no work for dead rows.
-// Group index and the staged first measure live in per-warp shared memory laid out
-// [row i][lane] (conflict-free for any mix of rows).  Dense RFOR probes look each run's value
-// up once and expand the payloads (runs share their key).  Grouped queries
-// pre-aggregate in a per-CTA shared-memory hash table (open addressing) and flush it once,
-// so hot groups (q4.1 has 35) do not serialise on global atomics.
+//    entry) -- no work for dead rows.
+// GPU-RFOR columns are evaluated in RUN space (rfor_col): a range or a probe once per run
+// (the rows of a run share its value) -- the run's passing bit reaches its rows
+// through one 64-bit add per thread -- and measures / group payloads per alive row through
+// the row's run number; the run expansion of the decode is never materialised.
+// The group index lives in per-warp shared memory laid out [row i][lane] (conflict-free for
+// any mix of rows).  The first of two measures stays in its ring item (held until the
+// round's last column aggregates) and is re-read per alive row; only a DFOR / RFOR first
+// measure is staged in a per-warp array.  Grouped queries pre-aggregate in a per-CTA
+// shared-memory hash table (open addressing) and flush it once, so hot groups (q4.1 has 35)
+// do not serialise on global atomics.
 struct StarArgs {
   int32_t role[TP_MAX_COLS], lo[TP_MAX_COLS], hi[TP_MAX_COLS];
   const int32_t* table[TP_MAX_COLS];
   int32_t key_min[TP_MAX_COLS];
   uint32_t table_len[TP_MAX_COLS], stride[TP_MAX_COLS];
   uint32_t gmode[TP_MAX_COLS];   // probe: 0 filter only, 1 group = p * stride (first), 2 group += p * stride
-  uint32_t mstage[TP_MAX_COLS];  // measure: 1 = the first of two (staged), 0 = the aggregating one
+  uint32_t mstage[TP_MAX_COLS];  // measure: 1 = the first of two, 0 = the aggregating one
   int agg;
   uint32_t ngroups;
   uint32_t gzero;                // grouped without payload probes: every row is group 0
-  uint32_t gs_off, ws_off;       // per-warp scratch offsets (words) of the group / staged-measure arrays
+  uint32_t hold_m1;              // the first measure is read back from its held ring item (FOR / None)
+  uint32_t gs_off, ws_off;       // per-warp scratch (words): group index, staged first measure (no hold)
+  uint32_t ra_off, sb_off;       // per-warp scratch: RFOR run array (1024), start / pass / alive words (3 x 33)
   uint32_t ht_slots, ht_shift;   // shared-memory aggregation table (grouped queries)
   uint32_t sparse_max;           // warp alive-row count at or below which a column is evaluated sparsely
   uint32_t sparse_lane_max;      // ... and the busiest lane's alive rows: the sparse loop runs for the
@@ -808,21 +997,24 @@ struct StarArgs {
 #define TP_HT_MAX_SLOTS 1024
 #endif
 constexpr uint32_t HT_MAX_SLOTS = TP_HT_MAX_SLOTS, HT_EMPTY = 0xffffffffu, HT_PROBES = 64;
-// slots: a power of two >= 2 x the dense group count (at most 2048); 4 words per slot:
+// slots: a power of two >= 2 x the dense group count (at most HT_MAX_SLOTS); 4 words per slot:
 // key, sum lo, sum hi, count
 static inline uint32_t ht_slots(uint32_t ngroups) {
   uint32_t s = 256;
   while (s < HT_MAX_SLOTS && s < 2u * ngroups) s <<= 1;
   return s;
 }
-
-#ifndef TP_STAR_SPIN
-#define TP_STAR_SPIN false
+constexpr uint32_t STAR_RA_WORDS = 1024, STAR_SB_WORDS = 3 * 33 + 1;
+#ifndef TP_STAR_RING_WORDS
+#define TP_STAR_RING_WORDS 8192u           // 32 KB
 #endif
+#ifndef TP_STAR_RING_WORDS_GROUPED
+#define TP_STAR_RING_WORDS_GROUPED 6144u   // 24 KB
+#endif
+
 template <uint32_t MASK, bool GROUPED>
 struct StarOp : OpBase {
   static constexpr uint32_t kMask = MASK;
-  static constexpr bool kProducerSpin = TP_STAR_SPIN;
   const StarArgs* A;
   uint64_t acc, cnt;  // ungrouped (q1.x): reduce in registers
   uint32_t alive;
@@ -831,6 +1023,9 @@ struct StarOp : OpBase {
   uint32_t* hhi;   // (a 64-bit shared atomicAdd is a CAS loop on sm_100)
   uint32_t* hcnt;
   uint32_t hmask, hshift;
+  // the held first measure: this thread's miniblock view (FOR) or row pointer (None)
+  const uint32_t* m1w;
+  uint32_t m1ref, m1b, m1none;
 
   __device__ void cta_init(const Params& P, uint32_t* smem) {
     if (GROUPED) {
@@ -872,7 +1067,13 @@ struct StarOp : OpBase {
   }
   __device__ void begin(const Params& P, const StageCtx& C, const Lane& g) { alive = valid_rows(P, C, g); }
 
-  // the role of column c applied to row i (value x) -- shared by both modes
+  // the first measure of row i (the held item, or the staged array)
+  __device__ __forceinline__ uint32_t m1_at(uint32_t i, const uint32_t* W, uint32_t lane) const {
+    if (!A->hold_m1) return W[32u * i + lane];
+    if ((MASK & M_NONE) && m1none) return none_at(m1w, m1b, i);
+    return m1ref + extract_at(m1w, i * m1b, __funnelshift_lc(0xffffffffu, 0u, m1b));
+  }
+  // the role of column c applied to row i (value x) -- shared by every mode
   __device__ __forceinline__ void apply_range(uint32_t c, uint32_t i, uint32_t x) {
     if ((uint32_t)((int32_t)x - A->lo[c]) > (uint32_t)(A->hi[c] - A->lo[c])) alive &= ~(1u << i);
   }
@@ -901,142 +1102,263 @@ struct StarOp : OpBase {
       for (int i = 0; i < 32; ++i) G[32u * i + lane] += p[i] * stride;
     }
   }
+  // measure role of row i: its own filter; the first measure is only filtered here (read back
+  // later), the aggregating one combines with it and aggregates
   __device__ __forceinline__ void apply_measure(uint32_t c, uint32_t i, uint32_t x, const uint32_t* G, uint32_t* W,
                                                 uint32_t lane) {
-    if ((uint32_t)((int32_t)x - A->lo[c]) > (uint32_t)(A->hi[c] - A->lo[c])) {  // the measure's own filter
+    if ((uint32_t)((int32_t)x - A->lo[c]) > (uint32_t)(A->hi[c] - A->lo[c])) {
       alive &= ~(1u << i);
       return;
     }
     if (A->mstage[c]) {
-      W[32u * i + lane] = x;
+      if (!A->hold_m1) W[32u * i + lane] = x;
       return;
     }
     int64_t y = (int32_t)x;
-    if (A->agg == TP_AGG_MUL) y *= (int64_t)(int32_t)W[32u * i + lane];
-    else if (A->agg == TP_AGG_SUB) y = (int64_t)(int32_t)W[32u * i + lane] - y;
+    if (A->agg == TP_AGG_MUL) y *= (int64_t)(int32_t)m1_at(i, W, lane);
+    else if (A->agg == TP_AGG_SUB) y = (int64_t)(int32_t)m1_at(i, W, lane) - y;
     if (GROUPED) ht_add(A->gzero ? 0u : G[32u * i + lane], y);
     else acc += (uint64_t)y;
   }
 
-  __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c, uint32_t) {
-    if (!__any_sync(FULL, alive != 0u)) return;  // nothing survives in this warp's rows: skip the decode
-    const int role = A->role[c];
+  // ---------------- GPU-RFOR in run space
+  // rows R .. R + L - 1 of the warp round hold an alive row (runs longer than 32 rows: assumed)
+  __device__ __forceinline__ static bool run_alive(const uint32_t* AW, uint32_t R, uint32_t L) {
+    if (L > 32u) return true;
+    const uint32_t w = R >> 5;
+    const uint64_t win = ((uint64_t)AW[w + 1] << 32) | AW[w];
+    return ((win >> (R & 31u)) & ((1ull << L) - 1ull)) != 0ull;
+  }
+  // one stream block pair (rows 512 h .. 512 h + 511 of the round), CC entries per lane and pass
+  template <int CC>
+  __device__ __forceinline__ void rfor_runs(const uint32_t* bV, const uint32_t* bL, uint32_t r, uint32_t h,
+                                            uint32_t c, bool range, bool per_run, bool need_ra, bool all_alive,
+                                            uint32_t* RA, uint32_t* SB, uint32_t* PB, const uint32_t* AW,
+                                            uint32_t lane) {
+    const uint32_t refV = bV[1], refL = bL[1];  // references (FOR on both arrays)
+    const uint4 wv = make_uint4(bV[2], bV[3], bV[4], bV[5]), wl = make_uint4(bL[2], bL[3], bL[4], bL[5]);
+    const int32_t* __restrict__ T = A->table[c];
+    const uint32_t kmin = (uint32_t)A->key_min[c], tlen = A->table_len[c];
+    const int32_t lo = A->lo[c];
+    const uint32_t span = (uint32_t)(A->hi[c] - lo);
+    uint32_t rowbase = 0u;  // rows of the block covered by earlier passes
+#pragma unroll 1
+    for (uint32_t e00 = 0; e00 < r; e00 += 32u * CC) {
+      const uint32_t e0 = e00 + CC * lane, m = (e0 >> 5) & 15u, pos = e0 & 31u;
+      const uint32_t bv = checked_bw(byte_of(wv, m)), bl = checked_bw(byte_of(wl, m));  // R2, R17
+      const uint32_t* mV = bV + 6 + bytes_before(wv, m);  // miniblocks before m are full (R17)
+      const uint32_t* mL = bL + 6 + bytes_before(wl, m);
+      const uint32_t mv = __funnelshift_lc(0xffffffffu, 0u, bv), ml = __funnelshift_lc(0xffffffffu, 0u, bl);
+      uint32_t len[CC], val[CC];
+      uint32_t run = 0u;
+#pragma unroll
+      for (int k = 0; k < CC; ++k) {  // run lengths (scan step 1)
+        len[k] = e0 + k < r ? refL + extract_at(mL, (pos + k) * bl, ml) : 0u;
+        run += len[k];
+      }
+      const uint32_t incl = warp_inclusive_scan(run, lane);
+      uint32_t S = 512u * h + rowbase + incl - run;  // round row of entry e0's run start
+      rowbase += __shfl_sync(FULL, incl, 31);
+#pragma unroll
+      for (int k = 0; k < CC; ++k) val[k] = refV + extract_at(mV, (pos + k) * bv, mv);
+      uint32_t pass = 0u;  // bit k: run k passes the column's role
+      if (per_run) {
+        if (range) {
+#pragma unroll
+          for (int k = 0; k < CC; ++k) pass |= ((uint32_t)((int32_t)val[k] - lo) <= span ? 1u : 0u) << k;
+        } else {
+          // probes: every live run's lookup in flight before any result is used
+          uint32_t Sk = S;
+#pragma unroll
+          for (int k = 0; k < CC; ++k) {
+            const uint32_t key = val[k] - kmin;
+            const bool live = e0 + k < r && key < tlen && (all_alive || run_alive(AW, Sk, len[k]));
+            val[k] = live ? (uint32_t)__ldg(T + key) : 0xffffffffu;  // payload, -1 = miss
+            Sk += len[k];
+          }
+#pragma unroll
+          for (int k = 0; k < CC; ++k) pass |= ((int32_t)val[k] >= 0 ? 1u : 0u) << k;
+        }
+      }
+#pragma unroll
+      for (int k = 0; k < CC; ++k) {
+        if (e0 + k < r) {
+          const uint32_t bit = 1u << (S & 31u);
+          atomicOr(&SB[S >> 5], bit);
+          if ((pass >> k) & 1u) atomicOr(&PB[S >> 5], bit);
+          if (need_ra) RA[512u * h + e0 + k] = val[k];  // run number e0 + k of block h
+        }
+        S += len[k];
+      }
+    }
+  }
+  __device__ void rfor_col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c,
+                           int role) {
     const Col& col = P.col[c];
-    const bool rfor = (MASK & M_RFOR) && col.scheme == S_RFOR;
-    const bool dfor = (MASK & M_DFOR) && col.scheme == S_DFOR;  // prefix sums: no random access
+    const StreamView vv = stream_view(P, col.s0, C, 0), vl = stream_view(P, col.s1, C, 1);
+    uint32_t* RA = scratch + A->ra_off;
+    uint32_t* SB = scratch + A->sb_off;  // run-start bits per lane word
+    uint32_t* PB = SB + 33;              // passing-run-start bits
+    uint32_t* AW = PB + 33;              // alive words (+ a zero word)
     uint32_t* G = scratch + A->gs_off;
     uint32_t* W = scratch + A->ws_off;
     const uint32_t lane = g.lane;
+    const bool range = role == TP_ROLE_RANGE;
+    const bool per_run = role != TP_ROLE_MEASURE;
+    const bool payload = GROUPED && role == TP_ROLE_PROBE && A->gmode[c];
+    const bool need_ra = !per_run || payload;
+    const bool all_alive = __all_sync(FULL, alive == FULL);
+    __syncwarp();  // the previous RFOR column's readers are done
+    SB[lane] = 0u;
+    PB[lane] = 0u;
+    AW[lane] = alive;
+    if (lane == 0) AW[32] = 0u;
+    __syncwarp();
+    const uint32_t live_lanes = __ballot_sync(FULL, alive != 0u);
+#pragma unroll 1
+    for (uint32_t h = 0; h < 2; ++h) {
+      const uint32_t tl = C.round_base + 2u * g.cw + h;
+      if (C.t0s + tl >= C.tile_end) break;                    // warp-uniform
+      if (((live_lanes >> (16u * h)) & 0xffffu) == 0u) continue;  // no alive row in this block
+      const uint32_t* bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
+      const uint32_t* bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
+      uint32_t r = bV[0];  // run / value count
+      if (r > 512u) {
+        tp_flag_error(4u);  // TP_DEVERR_RUNS
+        r = 512u;
+      }
+      if (r <= 128u) rfor_runs<4>(bV, bL, r, h, c, range, per_run, need_ra, all_alive, RA, SB, PB, AW, lane);
+      else rfor_runs<8>(bV, bL, r, h, c, range, per_run, need_ra, all_alive, RA, SB, PB, AW, lane);
+    }
+    __syncwarp();
+    const uint32_t sb = SB[lane], jj = lane & 15u;
+    if (per_run) {
+      // the passing bit of the run covering the row before this lane's first row: the status of
+      // the last run start at or before it, a 16-lane segmented scan (row 0 of a block starts a run)
+      const uint32_t pb = PB[lane];
+      uint32_t has = sb != 0u, st = has ? (pb >> (31u - __clz(sb))) & 1u : 0u;
+#pragma unroll
+      for (int d = 1; d < 16; d <<= 1) {
+        const uint32_t yh = __shfl_up_sync(FULL, has, d, 16), ys = __shfl_up_sync(FULL, st, d, 16);
+        if (jj >= (uint32_t)d && !has) { has = yh; st = ys; }
+      }
+      const uint32_t up = __shfl_up_sync(FULL, st, 1, 16);
+      const uint32_t cin = jj ? up : 0u;
+      // rows of passing runs: adding 1 right above each passing start (and above a virtual start
+      // at row -1 carrying cin) into the continuation mask carries through the run's rows
+      const uint64_t cont = (uint64_t)(~sb) << 1;
+      const uint64_t add = ((uint64_t)pb << 2) | ((uint64_t)cin << 1);
+      alive &= (uint32_t)(((cont + add) ^ cont) >> 2);
+    }
+    if (need_ra && __any_sync(FULL, alive != 0u)) {
+      // run number of row i = run starts in the block up to row i - 1 (popc prefix over 16 lanes)
+      const uint32_t cl = __popc(sb);
+      const uint32_t base = seg16_inclusive_scan(cl) - cl + 512u * (lane >> 4) - 1u;
+      uint32_t m = alive;
+      while (m) {
+        const uint32_t i = __ffs(m) - 1u;
+        m &= m - 1u;
+        const uint32_t x = RA[base + __popc(sb & (0xffffffffu >> (31u - i)))];
+        if (payload) apply_payload(c, i, (int32_t)x, G, lane);
+        else apply_measure(c, i, x, G, W, lane);
+      }
+    }
+  }
+
+  __device__ bool col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c, uint32_t) {
+    if (!__any_sync(FULL, alive != 0u)) return true;  // nothing survives in this warp's rows: skip the decode
+    const int role = A->role[c];
+    const Col& col = P.col[c];
+    if ((MASK & M_RFOR) && col.scheme == S_RFOR) {
+      rfor_col(P, C, g, scratch, c, role);
+      return true;
+    }
+    const bool dfor = (MASK & M_DFOR) && col.scheme == S_DFOR;  // prefix sums: no random access
+    const bool none = (MASK & M_NONE) && col.scheme == S_NONE;
+    const bool hold = A->hold_m1 && A->mstage[c];
+    uint32_t* G = scratch + A->gs_off;
+    uint32_t* W = scratch + A->ws_off;
+    const uint32_t lane = g.lane;
+    if (hold) {  // this thread's view of the first measure, read back when the last column aggregates
+      if (none) {
+        uint32_t sw;
+        m1w = none_row(P, col, C, g, sw);
+        m1b = sw;
+        m1none = 1u;
+      } else {
+        const StreamView sv = stream_view(P, col.s0, C, 0);
+        uint32_t tl;
+        bool tv;
+        const MbView mv = for_mb(P, col, C, g, sv, tl, tv);
+        m1w = mv.w;
+        m1ref = mv.ref;
+        m1b = mv.b;
+        m1none = 0u;
+      }
+    }
     const uint32_t nal = __reduce_add_sync(FULL, __popc(alive));
     const bool sparse =
         !dfor && ((nal <= A->sparse_max &&
                    // a FOR filter / measure decodes densely for a few instructions a row: it goes
-                   // sparse only if the busiest lane's rows are few too (probes and RFOR columns
-                   // save far more per skipped row: L2 lookups, run expansion)
-                   (role == TP_ROLE_PROBE || rfor || __reduce_max_sync(FULL, __popc(alive)) <= A->sparse_lane_max)) ||
+                   // sparse only if the busiest lane's rows are few too (probes save far more per
+                   // skipped row: L2 lookups)
+                   (role == TP_ROLE_PROBE || __reduce_max_sync(FULL, __popc(alive)) <= A->sparse_lane_max)) ||
                   (GROUPED && role == TP_ROLE_MEASURE && !A->mstage[c]));
-    RforChunk k;
-    uint32_t carry = 0u;
-    if (rfor) {
-      rfor_scatter_round(P, col, C, g, scratch);
-      k = rfor_chunk(scratch, lane);
-      if (!sparse && role == TP_ROLE_PROBE) {
-        // dense RFOR probe: one lookup per run -- the run-start values of this chunk become
-        // their payloads in place, and the expansion below spreads the payloads
-        const int32_t* __restrict__ T = A->table[c];
-        const uint32_t kmin = (uint32_t)A->key_min[c], len = A->table_len[c];
-        uint32_t mm = k.mask;
-        while (mm) {
-          uint32_t pos[4], key[4];
-          bool ok[4];
-#pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            ok[q] = mm != 0u;
-            pos[q] = rfor_a_pos(32u * k.j + (__ffs(mm) - 1u));
-            mm &= mm - 1u;
-            key[q] = ok[q] ? k.A[pos[q]] - kmin : 0xffffffffu;
-          }
-          int32_t pl[4];
-#pragma unroll
-          for (int q = 0; q < 4; ++q) pl[q] = key[q] < len ? __ldg(T + key[q]) : -1;
-#pragma unroll
-          for (int q = 0; q < 4; ++q)
-            if (ok[q]) k.A[pos[q]] = (uint32_t)pl[q];
-        }
-        __syncwarp();
-      }
-      carry = rfor_carry(k);
-    }
     if (!sparse) {
       // ---------------- dense: every row of the warp's round
       uint32_t v[32];
-      if (rfor) rfor_fill(k, carry, v);
-      else decode_col<MASK & ~M_RFOR, TP_QUERY_COMPACT>(P, c, C, g, scratch, v);
+      decode_col<MASK & ~M_RFOR, TP_QUERY_COMPACT>(P, c, C, g, scratch, v);
       if (role == TP_ROLE_RANGE) {
 #pragma unroll
         for (int i = 0; i < 32; ++i) apply_range(c, i, v[i]);
       } else if (role == TP_ROLE_PROBE) {
-        if (!rfor) {
-          // all 32 probes are issued before any result is used (32 L2 requests in flight)
-          const int32_t* __restrict__ T = A->table[c];
-          const uint32_t kmin = (uint32_t)A->key_min[c], len = A->table_len[c];
-          const uint32_t m = alive;
+        // all 32 probes are issued before any result is used (32 L2 requests in flight)
+        const int32_t* __restrict__ T = A->table[c];
+        const uint32_t kmin = (uint32_t)A->key_min[c], len = A->table_len[c];
+        const uint32_t m = alive;
 #pragma unroll
-          for (int i = 0; i < 32; ++i) {
-            const uint32_t kk = v[i] - kmin;
-            v[i] = ((m >> i) & 1u) && kk < len ? (uint32_t)__ldg(T + kk) : 0xffffffffu;
-          }
+        for (int i = 0; i < 32; ++i) {
+          const uint32_t kk = v[i] - kmin;
+          v[i] = ((m >> i) & 1u) && kk < len ? (uint32_t)__ldg(T + kk) : 0xffffffffu;
         }
         dense_payload(c, v, G, lane);
       } else {
-        // measure: its own filter, then stage it (first of two) or aggregate it (ungrouped;
-        // grouped aggregating measures always take the sparse path)
         const int32_t lo = A->lo[c];
         const uint32_t span = (uint32_t)(A->hi[c] - lo);
 #pragma unroll
         for (int i = 0; i < 32; ++i)
           if ((uint32_t)((int32_t)v[i] - lo) > span) alive &= ~(1u << i);
         if (A->mstage[c]) {
+          if (!hold) {
 #pragma unroll
-          for (int i = 0; i < 32; ++i) W[32u * i + lane] = v[i];
-        } else if (GROUPED) {
-          // only a DFOR aggregating measure gets here (others go sparse): its alive rows
-          uint32_t m = alive;
-          while (m) {
-            const uint32_t i = __ffs(m) - 1u;
-            m &= m - 1u;
-            int64_t y = (int32_t)v[i];
-            if (A->agg == TP_AGG_MUL) y *= (int64_t)(int32_t)W[32u * i + lane];
-            else if (A->agg == TP_AGG_SUB) y = (int64_t)(int32_t)W[32u * i + lane] - y;
-            ht_add(A->gzero ? 0u : G[32u * i + lane], y);
+            for (int i = 0; i < 32; ++i) W[32u * i + lane] = v[i];
           }
         } else {
+          // (grouped: only a DFOR aggregating measure gets here, the others go sparse) -- static
+          // row indices throughout: v[] stays in registers
           const uint32_t m = alive;
-          if (A->agg == TP_AGG_MUL) {
 #pragma unroll
-            for (int i = 0; i < 32; ++i)
-              if (m & (1u << i)) acc += (uint64_t)((int64_t)(int32_t)v[i] * (int32_t)W[32u * i + lane]);
-          } else {
-            const bool sub = A->agg == TP_AGG_SUB;
-#pragma unroll
-            for (int i = 0; i < 32; ++i) {
-              const int64_t y = sub ? (int64_t)(int32_t)W[32u * i + lane] - (int32_t)v[i] : (int64_t)(int32_t)v[i];
-              if (m & (1u << i)) acc += (uint64_t)y;
+          for (int i = 0; i < 32; ++i) {
+            if (m & (1u << i)) {
+              int64_t y = (int32_t)v[i];
+              if (A->agg == TP_AGG_MUL) y *= (int64_t)(int32_t)m1_at(i, W, lane);
+              else if (A->agg == TP_AGG_SUB) y = (int64_t)(int32_t)m1_at(i, W, lane) - y;
+              if (GROUPED) ht_add(A->gzero ? 0u : G[32u * i + lane], y);
+              else acc += (uint64_t)y;
             }
           }
         }
       }
-      return;
+      return !hold;
     }
     // ---------------- sparse: alive rows only, values read out of the staged tile
     MbView mv;
     uint32_t bmask = 0u, nsw = 0u;
-    const bool none = (MASK & M_NONE) && col.scheme == S_NONE;
     const uint32_t* nw = nullptr;
     if (none) {
       nw = none_row(P, col, C, g, nsw);
-    } else if (!rfor) {
-      const StreamView sv = stream_view(P, col.s0, C);
+    } else {
+      const StreamView sv = stream_view(P, col.s0, C, 0);
       uint32_t tl;
       bool tv;
       mv = for_mb(P, col, C, g, sv, tl, tv);
@@ -1051,9 +1373,7 @@ struct StarOp : OpBase {
         ok[q] = m != 0u;
         ii[q] = ok[q] ? __ffs(m) - 1u : 0u;
         m &= m - 1u;
-        xx[q] = none ? none_at(nw, nsw, ii[q])
-                : rfor ? rfor_row(k, carry, ii[q])
-                       : mv.ref + extract_at(mv.w, ii[q] * mv.b, bmask);  // Alg. 1, one entry
+        xx[q] = none ? none_at(nw, nsw, ii[q]) : mv.ref + extract_at(mv.w, ii[q] * mv.b, bmask);  // Alg. 1, one entry
       }
       if (role == TP_ROLE_RANGE) {
 #pragma unroll
@@ -1077,6 +1397,7 @@ struct StarOp : OpBase {
           if (ok[q]) apply_measure(c, ii[q], xx[q], G, W, lane);
       }
     }
+    return !hold;
   }
   __device__ void end(const Params&, const StageCtx&, const Lane&) {
     if (!GROUPED) cnt += __popc(alive);
@@ -1132,21 +1453,25 @@ __global__ void __launch_bounds__(THREADS, 3)
   op.out = out;
   op.acc = 0;
   op.alive = 0;
-  run_pipeline(P, op);
+  run_query_pipeline(P, op);
 }
 
-#ifndef TP_QUERY_MINB
-#define TP_QUERY_MINB 3
+// grouped queries: 3 CTAs / SM (the hash table and the group array); q1.x: 3 (at 4 the RFOR
+// run decode spills, measured in the ptxas report)
+#ifndef TP_STAR_MINB_UNGROUPED
+#define TP_STAR_MINB_UNGROUPED 3
 #endif
 template <uint32_t MASK, bool GROUPED>
-__global__ void __launch_bounds__(THREADS, TP_QUERY_MINB)
+__global__ void __launch_bounds__(THREADS, GROUPED ? 3 : TP_STAR_MINB_UNGROUPED)
     k_star_query(const __grid_constant__ Params P, const __grid_constant__ StarArgs A) {
   StarOp<MASK, GROUPED> op;
   op.A = &A;
   op.acc = 0;
   op.cnt = 0;
   op.alive = 0;
-  run_pipeline(P, op);
+  op.m1w = nullptr;
+  op.m1ref = op.m1b = op.m1none = 0u;
+  run_query_pipeline(P, op);
 }
 
 
@@ -1360,8 +1685,23 @@ static uint32_t align4(uint32_t w) { return (w + 3u) & ~3u; }
 // data region (TPR * rounds tiles of at most max_tile_words + alignment slop) and a
 // block_starts region; item size = the largest column's.  extra_scratch: words per
 // consumer warp (after the view table); agg_words: per-CTA aggregation table.
+// query pipeline: the largest ring item column k can produce (a range of TPR tiles: data words
+// + alignment + the unpack's over-read, block_starts words + alignment; None: one tensor box)
+static uint32_t query_item_words(const tp_column& k) {
+  if (k.scheme == TP_NONE) return TPR * TILE_ROWS + 256u;  // + the box's 1024-byte alignment
+  uint32_t w = 0;
+  for (int s = 0; s < (k.scheme == TP_RFOR ? 2 : 1); ++s) {
+    uint32_t mtw = s == 0 ? k.max_tile_words0 : k.max_tile_words1;
+    if (mtw == 0 || mtw > worst_tile_words(k.scheme)) mtw = worst_tile_words(k.scheme);
+    const uint32_t starts = k.scheme == TP_RFOR ? TPR + 1u : 4u * TPR + 1u;
+    w += align4(TPR * mtw + 6u) + 4u + align4(starts + 6u);
+  }
+  return w;
+}
+
 static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_scratch, uint32_t agg_words,
-                              Params& P, size_t& smem_bytes) {
+                              Params& P, size_t& smem_bytes, bool query = false, bool rfor_scratch = true,
+                              uint32_t ring_min_words = 0) {
   memset(&P, 0, sizeof(P));
   if (!cols || ncols < 1 || ncols > TP_MAX_COLS) return TP_EINVAL;
   const uint64_t n = cols[0].n;
@@ -1427,6 +1767,26 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
       ++P.nstreams;
     }
     max_round_words = std::max(max_round_words, rw);
+  }
+  if (query) {
+    // the byte ring of the query pipeline (run_query_pipeline): at least twice the largest item
+    uint32_t max_item = 0;
+    for (int c = 0; c < ncols; ++c) max_item = std::max(max_item, query_item_words(cols[c]));
+    P.rounds = 1;
+    P.ncols = (uint32_t)ncols;
+    P.n = (uint32_t)n;
+    P.ntiles = (uint32_t)((n + TILE_ROWS - 1) / TILE_ROWS);
+    P.ring_words = (std::max(ring_min_words, 2u * max_item) + 255u) & ~255u;
+    P.nstages = 0;
+    P.stage_words = 0;
+    P.staging_off = (any_rfor && rfor_scratch) ? RFOR_SCRATCH_WORDS : 0u;
+    P.scratch_words_per_warp = align4(P.staging_off + extra_scratch);
+    P.scratch_off = P.ring_words;
+    P.agg_off = P.scratch_off + CONSUMER_WARPS * P.scratch_words_per_warp;
+    P.bar_off = align4(P.agg_off + agg_words);
+    if (P.bar_off & 1u) ++P.bar_off;
+    smem_bytes = (size_t)P.bar_off * 4 + 2 * QNS * 8 + QNS * 16 + 16;
+    return TP_OK;
   }
   // rounds per item: single-column kernels carry ~16 KB of compressed words per item
   // (bytes in flight at low bitwidths, where one round is a few hundred bytes); queries
@@ -1634,7 +1994,7 @@ tp_status tp_select_project_sum(const tp_column* dcols, int ncols, const int32_t
   }
   Params P;
   size_t smem = 0;
-  tp_status st = build_params(ord, k, 0, 0, P, smem);
+  tp_status st = build_params(ord, k, 0, 0, P, smem, true, true, TP_STAR_RING_WORDS);
   if (st != TP_OK) return st;
   auto out = reinterpret_cast<unsigned long long*>(d_result);
   const int cap = (int)((P.ntiles + 1) / 2);
@@ -1701,13 +2061,40 @@ tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int nc
   if (const char* e = getenv("TILEPACK_SPARSE_LANE_MAX")) A.sparse_lane_max = (uint32_t)atoi(e);  // tuning
   if (const char* e = getenv("TILEPACK_SPARSE_MAX")) A.sparse_max = (uint32_t)atoi(e);  // tests: force a mode
   const uint32_t hts = grouped ? ht_slots(ngroups) : 0u;
-  const uint32_t gwords = grouped ? 32u * 32u : 0u, wwords = nmeas == 2 ? 32u * 32u : 0u;
+  // byte ring: 24 KB next to the grouped queries' hash table and group arrays (3 CTAs / SM),
+  // 32 KB for q1.x (4 CTAs / SM); at least twice the largest item either way
+  const uint32_t ring_min = grouped ? TP_STAR_RING_WORDS_GROUPED : TP_STAR_RING_WORDS;
+  bool any_rfor = false;
+  uint32_t mx = 0;
+  for (int c = 0; c < ncols; ++c) {
+    any_rfor |= dcols[c].scheme == TP_RFOR;
+    mx = std::max(mx, query_item_words(dcols[c]));
+  }
+  const uint32_t ring = (std::max(ring_min, 2u * mx) + 255u) & ~255u;
+  // the first measure stays in its ring item until the last column aggregates (no staging array)
+  // when it is random-access (FOR / None) and the items from it to the last column always fit
+  // in the ring next to one item of wrap-around waste
+  bool hold = false;
+  for (int c = 0; c < ncols - 1; ++c) {
+    if (roles[c].role != TP_ROLE_MEASURE) continue;
+    if (dcols[c].scheme == TP_FOR || dcols[c].scheme == TP_NONE) {
+      uint32_t span = 0;
+      for (int q = c; q < ncols; ++q) span += query_item_words(dcols[q]);
+      hold = span + mx <= ring;
+    }
+  }
+  if (const char* e = getenv("TILEPACK_STAR_NO_HOLD")) hold = hold && atoi(e) == 0;  // tests: the staged path
+  const uint32_t gwords = grouped ? 32u * 32u : 0u, wwords = nmeas == 2 && !hold ? 32u * 32u : 0u;
+  const uint32_t rwords = any_rfor ? STAR_RA_WORDS + STAR_SB_WORDS : 0u;
   Params P;
   size_t smem = 0;
-  tp_status st = build_params(dcols, ncols, gwords + wwords, 4u * hts, P, smem);
+  tp_status st = build_params(dcols, ncols, gwords + wwords + rwords, 4u * hts, P, smem, true, false, ring_min);
   if (st != TP_OK) return st;
-  A.gs_off = P.staging_off;
-  A.ws_off = P.staging_off + gwords;
+  A.hold_m1 = hold ? 1u : 0u;
+  A.gs_off = 0;
+  A.ws_off = gwords;
+  A.ra_off = gwords + wwords;
+  A.sb_off = A.ra_off + STAR_RA_WORDS;
   A.ht_slots = hts;
   A.ht_shift = 32u - (uint32_t)__builtin_ctz(hts ? hts : 1u);
   A.sums = reinterpret_cast<long long*>(d_sums);

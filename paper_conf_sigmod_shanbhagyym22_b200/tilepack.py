@@ -311,7 +311,8 @@ def tp_bench_int_roof(kind: int, iters: int, d_sink, stream=None) -> int:
 
 
 INT_ROOF_KINDS = {0: "SHF", 1: "LOP3", 2: "IADD3", 3: "IMAD", 4: "SHF+LOP3+IADD3 (ALU pipe)",
-                  5: "LOP3+IMAD (ALU+FMA pipes)"}
+                  5: "LOP3+IMAD (ALU+FMA pipes)", 6: "SHF imm", 7: "LOP3 imm", 8: "IMAD imm",
+                  9: "LOP3+SHF+IMAD imm (ALU+FMA pipes)"}
 
 
 def measure_int_roof(iters: int = 4000, reps: int = 5, stream=None) -> dict:
@@ -334,6 +335,7 @@ def measure_int_roof(iters: int = 4000, reps: int = 5, stream=None) -> dict:
             best = ms if best is None or ms < best else best
         out[name] = {"warp_insts": w, "ms": best, "warp_insts_per_s": w / (best / 1e3),
                      "lane_ops_per_s": 32 * w / (best / 1e3)}
+    out["roof_warp_insts_per_s"] = max(v["warp_insts_per_s"] for v in out.values())
     return out
 
 

@@ -89,3 +89,40 @@ def test_two_rank_gloo_combine_equals_unsharded():
             assert out[r][scheme] == [oracle.column_sum(x), n], (scheme, r)
     want = oracle.select_project_sum(list(cols.values()), [0, 0, 0], [4000, 2**31 - 1, 30000], "mul", 0, 2)
     assert out[0]["query"] == out[1]["query"] == want
+
+
+def _ssb_worker(rank, port, sf, out):
+    """bench.py's SSB leg on one rank, with the oracle as the per-rank kernel: the rank generates
+    ONLY its 512-row tile range of lineorder (datagen.ssb rows=, as bench.ssb_leg does), answers
+    every query on it, and the dense per-group partials are combined with one allreduce each."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=WORLD)
+    try:
+        import datagen.ssb as gen
+        from oracle import ssb as ossb
+        total = gen.num_rows(sf, seed=5000)
+        r0, r1 = tpd.tile_range(total, rank, WORLD)
+        db = gen.generate(sf, seed=5000, columns=gen.QUERY_COLUMNS, rows=(r0, r1))
+        assert len(db["lineorder"]["lo_orderdate"]) == r1 - r0
+        whole = ossb.SSB(gen.generate(sf, seed=5000, columns=gen.QUERY_COLUMNS))
+        part = ossb.SSB(db)
+        res = {}
+        for q in ossb.QUERIES:
+            want = whole.run(q)
+            keys = [tuple(r[:-1]) for r in want]           # the group space, identical on every rank
+            got = {tuple(r[:-1]): r[-1] for r in part.run(q)}
+            assert set(got) - set(keys) <= {()}, q           # a shard never invents a group
+            dense = torch.tensor([got.get(k, 0) for k in keys], dtype=torch.int64)
+            tpd.combine([dense])                             # the GPU path's allreduce of partials
+            res[q] = [list(k) + [int(v)] for k, v in zip(keys, dense.tolist())] == [list(r) for r in want]
+        out[rank] = res
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.timeout(600)
+def test_two_rank_gloo_ssb_leg_equals_unsharded():
+    out = mp.Manager().dict()
+    mp.spawn(_ssb_worker, args=(_free_port(), 0.05, out), nprocs=WORLD, join=True)
+    for r in range(WORLD):
+        assert all(out[r].values()), out[r]

@@ -157,7 +157,7 @@ def test_device_format_errors_flagged():
     byte > 32 (R3, R5) and a max_tile_words below the column's real tile span (the ring stays in
     bounds, the flag says the result is undefined)."""
     assert tp.tp_device_errors() == 0
-    x = datagen.uniform_bits(10, 512 * 64 + 5, seed=3)
+    x = datagen.uniform_bits(10, 5_000_000 + 5, seed=3)  # many tiles per CTA: items of many tiles
     h = tp.encode(x, "for")
     d = h.to_device()
     tp.decode_sum(d)

@@ -25,7 +25,9 @@ def _inputs(seed):
     srt = datagen.near_sorted(N, seed=seed + 1)                 # DFOR column
     t1 = np.where(rng.random(3000) < 0.3, rng.integers(0, 7, 3000), -1).astype(np.int32)
     t2 = np.where(rng.random(2000) < 0.5, rng.integers(0, 25, 2000), -1).astype(np.int32)
-    return dict(keys=keys, fk=fk, qty=qty, price=price, cost=cost, srt=srt, t1=t1, t2=t2)
+    short = (datagen.runs(N, 1, seed=seed + 2) % 3000).astype(np.int32)   # RFOR, 512 runs per block
+    long_ = (datagen.runs(N, 100, seed=seed + 3) % 3000).astype(np.int32)  # RFOR, runs across many lanes
+    return dict(keys=keys, fk=fk, qty=qty, price=price, cost=cost, srt=srt, t1=t1, t2=t2, short=short, long=long_)
 
 
 def _cases(d):
@@ -57,6 +59,24 @@ def _cases(d):
         # grouped MUL, filter-only probe, no payload probe -> single group 0 of 3
         (["fk", "qty", "cost"], ["for", "for", "for"],
          [dict(role="probe", table=d["t2"], key_min=0, stride=0), meas(), meas(0, 60000)], "mul", 3),
+        # grouped, the aggregating measure GPU-DFOR (dense path, no random access)
+        (["fk", "srt"], ["for", "dfor"], [probe2, meas(lo_s, hi_s)], "sum", 25),
+        # grouped, the aggregating measure GPU-RFOR (per alive row through its run number)
+        (["fk", "keys"], ["for", "rfor"], [probe2, meas(100, 2000)], "sum", 25),
+        # the first measure GPU-RFOR (staged per row), FOR range, FOR aggregating product
+        (["keys", "qty", "price"], ["rfor", "for", "for"], [meas(0, 2500), dict(role="range", lo=1, hi=30), meas()],
+         "mul", 1),
+        # RFOR with one-row runs (512 runs per block: two passes of 8 entries per lane) as a range,
+        # RFOR with runs of up to 199 rows (spanning lanes and blocks) as a grouped probe
+        (["short", "long", "price"], ["rfor", "rfor", "for"],
+         [dict(role="range", lo=0, hi=2000), dict(role="probe", table=d["t1"], key_min=0, stride=25), meas()],
+         "sum", 7 * 25),
+        # RFOR range first, a held None first measure, a FOR probe, grouped difference
+        (["keys", "price", "fk", "cost"], ["rfor", "none", "for", "for"],
+         [dict(role="range", lo=0, hi=1500), meas(), probe2, meas()], "sub", 25),
+        # ungrouped RFOR probe (filter only) on one-row runs, held FOR first measure, product
+        (["short", "cost", "price"], ["rfor", "for", "for"],
+         [dict(role="probe", table=d["t1"], key_min=0, stride=0), meas(0, 90000), meas()], "mul", 1),
     ]
 
 
@@ -87,8 +107,9 @@ def test_oracle_star_query_brute_force():
 
 
 @pytest.mark.gpu
+@pytest.mark.parametrize("hold", ["hold", "staged"])
 @pytest.mark.parametrize("mode", ["dense", "sparse", "auto"])
-def test_gpu_star_query_modes(mode, monkeypatch):
+def test_gpu_star_query_modes(mode, hold, monkeypatch):
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
@@ -96,7 +117,34 @@ def test_gpu_star_query_modes(mode, monkeypatch):
     if mode != "auto":
         monkeypatch.setenv("TILEPACK_SPARSE_MAX", "0" if mode == "dense" else "1024")
         monkeypatch.setenv("TILEPACK_SPARSE_LANE_MAX", "0" if mode == "dense" else "32")
-    for seed in (1, 2):
+    if hold == "staged":  # the first measure staged per row instead of read back from its ring item
+        monkeypatch.setenv("TILEPACK_STAR_NO_HOLD", "1")
+    _run_cases(torch, tp, N, (1, 2), mode)
+
+
+@pytest.mark.gpu
+def test_gpu_star_query_long_columns():
+    """20M rows: every CTA runs tens of rounds, so the byte ring wraps many times with items of
+    very different sizes (RFOR 6-bit keys next to 25-bit FOR prices) and held first measures."""
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sigmod_shanbhagyym22_b200 import tilepack as tp
+    _run_cases(torch, tp, 20_000_000 + 333, (3,), "auto")
+    assert tp.tp_device_errors() == 0
+
+
+def _run_cases(torch, tp, n, seeds, mode):
+    global N
+    n0, N = N, n
+    try:
+        _run_cases_n(torch, tp, seeds, mode)
+    finally:
+        N = n0
+
+
+def _run_cases_n(torch, tp, seeds, mode):
+    for seed in seeds:
         d = _inputs(seed)
         dev = {}
         for ci, (names, schemes, roles, agg, G) in enumerate(_cases(d)):
@@ -122,3 +170,4 @@ def test_gpu_star_query_modes(mode, monkeypatch):
             want_s, want_c = oracle.star_query([d[nm] for nm in names], roles, agg, G)
             assert np.array_equal(sums.cpu().numpy(), want_s), (mode, seed, ci)
             assert np.array_equal(cnts.cpu().numpy(), want_c), (mode, seed, ci)
+    assert tp.tp_device_errors() == 0
