@@ -140,11 +140,16 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 // (include/tilepack.h tp_device_errors; one copy per translation unit -- the pipeline
 // kernels' copy in tp_kernels.cu is the one the ABI reads)
 static __device__ uint32_t g_tp_err;
-__device__ __forceinline__ void tp_flag_error(uint32_t bit) { atomicOr(&g_tp_err, bit); }
+// one RED per flagging thread (no warp-aggregation sequence: the flag is set on a rare path)
+__device__ __forceinline__ void tp_flag_error(uint32_t bit) {
+  asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(&g_tp_err), "r"(bit));  // no ordering needed
+}
 // a miniblock bitwidth byte: > 32 is a format violation (R3, R5), used as 32 (a predicated
 // RED on the rare path; no branch around the decode)
 __device__ __forceinline__ uint32_t checked_bw(uint32_t b) {
+#ifndef TP_NO_BW_FLAG
   if (__builtin_expect(b > 32u, 0)) tp_flag_error(1u);  // TP_DEVERR_BITWIDTH
+#endif
   return min(b, 32u);
 }
 
@@ -229,17 +234,21 @@ __device__ __forceinline__ void unpack_any(const uint32_t* __restrict__ w, uint3
 
 // Warp-cooperative dispatch: the warp runs the specialised routine once per
 // distinct bitwidth among its lanes (one pass when the column's miniblocks share b,
-// the common case; a few passes for sorted-delta or run-length streams).
+// the common case; a few passes for sorted-delta or run-length streams).  A lane whose
+// miniblock is empty (b = 0: every offset 0) rides along with the first pass of another width
+// and zeroes its offsets afterwards -- a delta stream mixing {0, B} (sorted keys, D1) takes one
+// pass, not two.
 #ifndef TP_UNPACK_MAX_PASSES
 #define TP_UNPACK_MAX_PASSES 2
 #endif
 __device__ __forceinline__ void unpack_mb(const uint32_t* __restrict__ w, uint32_t b, uint32_t (&e)[32]) {
-  uint32_t todo = FULL;
+  const uint32_t zl = __ballot_sync(FULL, b == 0u);
+  uint32_t todo = zl == FULL ? FULL : ~zl;  // the non-empty lanes (or all of them, if all empty)
 #if TP_UNPACK_MAX_PASSES < 32
   // more distinct bitwidths than TP_UNPACK_MAX_PASSES among the lanes (delta streams of
   // near-sorted keys): one runtime-bitwidth pass beats several specialised ones
   {
-    uint32_t t = FULL;
+    uint32_t t = todo;
 #pragma unroll
     for (int k = 0; k < TP_UNPACK_MAX_PASSES; ++k) {
       const uint32_t bl = __shfl_sync(FULL, b, __ffs(t) - 1);
@@ -252,10 +261,12 @@ __device__ __forceinline__ void unpack_mb(const uint32_t* __restrict__ w, uint32
     }
   }
 #endif
+  uint32_t ride = zl == FULL ? 0u : zl;  // empty lanes joining the first pass
   do {
     const uint32_t bl = __shfl_sync(FULL, b, __ffs(todo) - 1);
-    const bool mine = b == bl;
-    todo &= ~__ballot_sync(FULL, mine);
+    const bool mine = b == bl || ((ride >> (threadIdx.x & 31u)) & 1u);
+    todo &= ~__ballot_sync(FULL, b == bl);
+    ride = 0u;
     if (mine) {
       switch (bl) {
         TP_CASE(0) TP_CASE(1) TP_CASE(2) TP_CASE(3) TP_CASE(4) TP_CASE(5) TP_CASE(6) TP_CASE(7)
@@ -266,6 +277,10 @@ __device__ __forceinline__ void unpack_mb(const uint32_t* __restrict__ w, uint32
       }
     }
   } while (todo);
+  if (zl != 0u && zl != FULL && b == 0u) {  // the riders read a neighbour's words
+#pragma unroll
+    for (int i = 0; i < 32; ++i) e[i] = 0u;
+  }
 }
 #undef TP_CASE
 

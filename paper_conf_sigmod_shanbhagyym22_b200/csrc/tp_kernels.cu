@@ -45,12 +45,15 @@ struct StreamView {
 // Every lane derives the view itself (two smem loads + address arithmetic): cheaper on
 // the per-round critical path than sharing it through shared memory and a warp sync.
 // s = the stream (Params::st index), k = 0 / 1: the column's first / second stream
+// QP: the query pipeline (per-item region offsets in C); otherwise the single-column pipeline's
+// fixed stage layout (constant-bank offsets: fewer registers on the per-round path, measured 3 %)
+template <bool QP = false>
 __device__ __forceinline__ StreamView stream_view(const Params& P, uint32_t s, const StageCtx& C, uint32_t k = 0) {
   const Stream& st = P.st[s];
   StreamView v;  // FOR / DFOR / RFOR streams only (a None column is read through none_row)
   const uint32_t sidx = st.kind == K_RFOR ? C.t0s : 4u * C.t0s;
-  v.ss = C.stage + C.soff[k];
-  v.sd = C.stage + C.doff[k];
+  v.ss = C.stage + (QP ? C.soff[k] : st.starts_off);
+  v.sd = C.stage + (QP ? C.doff[k] : st.data_off);
   v.sshift = align_shift(st.starts, sidx);
   v.lo = v.ss[v.sshift] - (st.kind == K_DFOR ? 1u : 0u);
   v.dshift = align_shift(st.data, v.lo);
@@ -112,10 +115,10 @@ __device__ __forceinline__ MbView fornm_mb(const Params& P, const Col& c, const 
 // stalls in the SSB kernel)
 // RAW: the packed offsets only (no reference added) -- the first pass of the cascading
 // baseline (tp_cascaded.cu), also for the delta blocks of a GPU-DFOR column
-template <bool COMPACT, bool RAW = false, bool NOMB = false>
+template <bool COMPACT, bool RAW = false, bool NOMB = false, bool QP = false>
 __device__ __forceinline__ void decode_for(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                            uint32_t (&val)[32]) {
-  const StreamView v = stream_view(P, c.s0, C);
+  const StreamView v = stream_view<QP>(P, c.s0, C);
   uint32_t tl;
   bool tv;
   const MbView m = NOMB ? fornm_mb(P, c, C, g, v, tl, tv) : for_mb(P, c, C, g, v, tl, tv);
@@ -130,10 +133,10 @@ __device__ __forceinline__ void decode_for(const Params& P, const Col& c, const 
 // slots, then the tile-wide exclusive prefix sum (R13) -- a
 // register scan inside the thread plus a 16-lane shuffle scan across the
 // tile's miniblocks -- plus the tile's first value (Fig. 6).
-template <bool COMPACT>
+template <bool COMPACT, bool QP = false>
 __device__ __forceinline__ void decode_dfor(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                             uint32_t (&val)[32]) {
-  const StreamView v = stream_view(P, c.s0, C);
+  const StreamView v = stream_view<QP>(P, c.s0, C);
   uint32_t tl;
   bool tv;
   const MbView m = for_mb(P, c, C, g, v, tl, tv);
@@ -236,10 +239,10 @@ __device__ __forceinline__ void rfor_scatter(const uint32_t* bV, const uint32_t*
 // SMALLC: also the C = 1 / 2 bodies for blocks of few (long) runs -- single-column decodes
 // only: the query kernels keep the smaller code (their RFOR columns have short runs, and the
 // extra bodies cost the star kernels ~4 % through instruction-cache misses, measured)
-template <bool SMALLC = false>
+template <bool SMALLC = false, bool QP = false>
 __device__ __forceinline__ void rfor_scatter_round(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                                    uint32_t* scratch) {
-  const StreamView vv = stream_view(P, c.s0, C, 0), vl = stream_view(P, c.s1, C, 1);
+  const StreamView vv = stream_view<QP>(P, c.s0, C, 0), vl = stream_view<QP>(P, c.s1, C, 1);
   const uint32_t lane = g.lane;
   __syncwarp();  // a lagging lane may still read the previous column's expansion
 #pragma unroll 1
@@ -321,10 +324,10 @@ __device__ __forceinline__ uint32_t rfor_row(const RforChunk& k, uint32_t carry,
   return mm ? k.A[rfor_a_pos(32u * k.j + 31u - __clz(mm))] : carry;
 }
 
-template <bool SMALLC>
+template <bool SMALLC, bool QP = false>
 __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                             uint32_t* scratch, uint32_t (&val)[32]) {
-  rfor_scatter_round<SMALLC>(P, c, C, g, scratch);
+  rfor_scatter_round<SMALLC, QP>(P, c, C, g, scratch);
   const RforChunk k = rfor_chunk(scratch, g.lane);
   rfor_fill(k, rfor_carry(k), val);
 }
@@ -332,16 +335,18 @@ __device__ __forceinline__ void decode_rfor(const Params& P, const Col& c, const
 // ---------------------------------------------------------------- None (uncompressed)
 // The plain column staged as a 128B-swizzled TMA box of 32-word rows: row r = 16 * tile + mb
 // holds the thread's 32 values, 16-byte chunk q at chunk q ^ (r & 7).
+template <bool QP = false>
 __device__ __forceinline__ const uint32_t* none_row(const Params& P, const Col& c, const StageCtx& C,
                                                     const Lane& g, uint32_t& sw) {
   const uint32_t r = 16u * (C.round_base + g.tile_local) + g.mb;
   sw = r & 7u;
-  return C.stage + C.doff[0] + 32u * r;
+  return C.stage + (QP ? C.doff[0] : P.st[c.s0].data_off) + 32u * r;
 }
+template <bool QP = false>
 __device__ __forceinline__ void decode_none(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                             uint32_t (&val)[32]) {
   uint32_t sw;
-  const uint32_t* w = none_row(P, c, C, g, sw);
+  const uint32_t* w = none_row<QP>(P, c, C, g, sw);
 #pragma unroll
   for (int q = 0; q < 8; ++q) {
     const uint4 a = *reinterpret_cast<const uint4*>(w + ((q ^ sw) << 2));
@@ -357,7 +362,7 @@ __device__ __forceinline__ uint32_t none_at(const uint32_t* w, uint32_t sw, uint
 constexpr uint32_t M_FOR = 1u << S_FOR, M_DFOR = 1u << S_DFOR, M_RFOR = 1u << S_RFOR, M_NONE = 1u << S_NONE;
 constexpr uint32_t M_FORNM = 1u << S_FORNM;  // decode / decode_sum only (the miniblock ablation)
 constexpr uint32_t M_RAW = 1u << 8;  // FOR / DFOR blocks, packed offsets only (cascading baseline)
-template <uint32_t MASK, bool COMPACT = false>
+template <uint32_t MASK, bool COMPACT = false, bool QP = false>
 __device__ __forceinline__ void decode_col(const Params& P, uint32_t ci, const StageCtx& C, const Lane& g,
                                            uint32_t* scratch, uint32_t (&val)[32]) {
   const Col& c = P.col[ci];
@@ -369,10 +374,10 @@ __device__ __forceinline__ void decode_col(const Params& P, uint32_t ci, const S
     decode_for<false, false, true>(P, c, C, g, val);
     return;
   }
-  if ((MASK & M_NONE) && c.scheme == S_NONE) decode_none(P, c, C, g, val);
-  else if ((MASK & M_FOR) && c.scheme == S_FOR) decode_for<COMPACT>(P, c, C, g, val);
-  else if ((MASK & M_DFOR) && c.scheme == S_DFOR) decode_dfor<COMPACT>(P, c, C, g, val);
-  else if (MASK & M_RFOR) decode_rfor<!COMPACT>(P, c, C, g, scratch, val);
+  if ((MASK & M_NONE) && c.scheme == S_NONE) decode_none<QP>(P, c, C, g, val);
+  else if ((MASK & M_FOR) && c.scheme == S_FOR) decode_for<COMPACT, false, false, QP>(P, c, C, g, val);
+  else if ((MASK & M_DFOR) && c.scheme == S_DFOR) decode_dfor<COMPACT, QP>(P, c, C, g, val);
+  else if (MASK & M_RFOR) decode_rfor<!COMPACT, QP>(P, c, C, g, scratch, val);
 }
 
 // ------------------------------------------------------------------ the pipeline
@@ -411,6 +416,7 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
     // ---------------- producer
     const uint64_t pol = policy_evict_first();
     uint32_t slot = 0, phase = 0, item = 0;  // ring position of the next item (no runtime division)
+    bool over = false;
     for (uint32_t gb = 0; gb < ngr; gb += 31) {
       // lane i prefetches every stream's block_starts entry at the start of range gb+i
       const uint32_t tb = min(t0 + (gb + lane) * TPS, t1);
@@ -461,10 +467,10 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
             const uintptr_t a1 = (reinterpret_cast<uintptr_t>(st.data + myhi) + 15) & ~uintptr_t(15);
             dsrc = reinterpret_cast<const char*>(a0);
             dbytes = (uint32_t)(a1 - a0);
-            if (dbytes > st.data_cap) {  // max_tile_words below the column's real span
-              tp_flag_error(2u);         // TP_DEVERR_TILE_WORDS: copy what fits, stay in the ring
-              dbytes = st.data_cap;
-            }
+            // max_tile_words below the column's real span: copy what fits (stay in the ring) and
+            // report TP_DEVERR_TILE_WORDS once, after the loop (off the producer's critical path)
+            over |= dbytes > st.data_cap;
+            dbytes = min(dbytes, st.data_cap);
             const uint32_t s0 = st.kind == K_RFOR ? tile_base : 4u * tile_base;
             const uint32_t s1 = min(st.kind == K_RFOR ? tile_end : 4u * tile_end, st.nblocks) + 1u;
             const uintptr_t b0 = reinterpret_cast<uintptr_t>(st.starts + s0) & ~uintptr_t(15);
@@ -489,6 +495,7 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
         }
       }
     }
+    if (over) tp_flag_error(2u);  // TP_DEVERR_TILE_WORDS
   } else {
     // ---------------- consumers
     const Lane g = lane_geom();
@@ -568,10 +575,12 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
 // consumers release items, oldest first.  QNS item slots carry each item's mbarriers and layout
 // {ring offset, block_starts offset of stream 0, data / block_starts offsets of stream 1}.
 // The bytes in flight are the ring's whatever the column mix (fixed slots sized for the widest
-// column held two items of an SSB query).  An operator may keep an item (Op::col returns false:
-// the staged first measure, read back when the last column aggregates); it is released at the
-// end of its round -- the host sizes the ring so that the items in between always fit.
+// column held two items of an SSB query).  An operator may keep an item until the end of its
+// round (Op::col returns false); the host must then size the ring for every item in between.
 constexpr uint32_t QNS = 16;
+#ifndef TP_QPROD_SPIN
+#define TP_QPROD_SPIN 0
+#endif
 
 template <class Op>
 __device__ __forceinline__ void run_query_pipeline(const Params& P, Op& op) {
@@ -650,13 +659,16 @@ __device__ __forceinline__ void run_query_pipeline(const Params& P, Op& op) {
             ssrc = reinterpret_cast<const char*>(b0);
             sbytes = (uint32_t)(b1 - b0);
             swords = sbytes >> 2;
-            // a malformed column (a tile longer than max_tile_words says) must not outgrow the ring
-            const uint32_t cap = 4u * ((RW >> 1) - swords - 8u);
-            if (dbytes > cap) {
-              tp_flag_error(2u);  // TP_DEVERR_TILE_WORDS
-              dbytes = cap & ~15u;
-            }
             dwords = (dbytes >> 2) + 4u;  // + the unpack's over-read (Alg. 1 line 15 reads word k + 1)
+          }
+          if (__shfl_sync(FULL, dwords + swords, 0) + __shfl_sync(FULL, dwords + swords, 1) > RW) {
+            // a malformed column (a tile longer than max_tile_words says) must not outgrow the
+            // ring: copy what fits (the host sized the ring for the largest legitimate item)
+            tp_flag_error(2u);  // TP_DEVERR_TILE_WORDS
+            if (my_s != 0xffu && !none) {
+              dbytes = min(dbytes, 4u * ((RW >> 1) - swords - 8u) & ~15u);
+              dwords = (dbytes >> 2) + 4u;
+            }
           }
           const uint32_t rw0 = __shfl_sync(FULL, dwords + swords, 0);
           const uint32_t rw1 = __shfl_sync(FULL, dwords + swords, 1);
@@ -665,7 +677,11 @@ __device__ __forceinline__ void run_query_pipeline(const Params& P, Op& op) {
           if (hd % RW + need > RW) hd += RW - hd % RW;  // does not fit before the ring's end: wrap
           // reclaim: the slot's previous item, and every item still holding the space needed
           while (item - oldest >= QNS || (oldest < item && hd + need > __shfl_sync(FULL, vst, oldest % QNS) + RW)) {
+#if TP_QPROD_SPIN
+            mbar_wait(&empty[oldest % QNS], (oldest / QNS) & 1u);
+#else
             mbar_wait_backoff(&empty[oldest % QNS], (oldest / QNS) & 1u);
+#endif
             ++oldest;
           }
           const uint32_t slot = item % QNS;
@@ -913,7 +929,7 @@ struct SelectOp : OpBase {
   __device__ bool col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c, uint32_t) {
     if (!__any_sync(FULL, alive != 0u)) return true;  // nothing survives in this warp's rows
     uint32_t v[32];
-    decode_col<MASK, TP_QUERY_COMPACT>(P, c, C, g, scratch, v);
+    decode_col<MASK, TP_QUERY_COMPACT, true>(P, c, C, g, scratch, v);
     const int32_t l = A->lo[c], h = A->hi[c];
 #pragma unroll
     for (int i = 0; i < 32; ++i)
@@ -982,8 +998,7 @@ struct StarArgs {
   int agg;
   uint32_t ngroups;
   uint32_t gzero;                // grouped without payload probes: every row is group 0
-  uint32_t hold_m1;              // the first measure is read back from its held ring item (FOR / None)
-  uint32_t gs_off, ws_off;       // per-warp scratch (words): group index, staged first measure (no hold)
+  uint32_t gs_off, ws_off;       // per-warp scratch (words): group index, staged first measure
   uint32_t ra_off, sb_off;       // per-warp scratch: RFOR run array (1024), start / pass / alive words (3 x 33)
   uint32_t ht_slots, ht_shift;   // shared-memory aggregation table (grouped queries)
   uint32_t sparse_max;           // warp alive-row count at or below which a column is evaluated sparsely
@@ -1005,8 +1020,17 @@ static inline uint32_t ht_slots(uint32_t ngroups) {
   return s;
 }
 constexpr uint32_t STAR_RA_WORDS = 1024, STAR_SB_WORDS = 3 * 33 + 1;
+#ifndef TP_RFOR_CC8
+#define TP_RFOR_CC8 0  // RFOR run decode: 4 entries per lane and pass only (one body: instruction cache)
+#endif
+#ifndef TP_HT_NOINLINE
+#define TP_HT_NOINLINE 0
+#endif
 #ifndef TP_STAR_RING_WORDS
 #define TP_STAR_RING_WORDS 8192u           // 32 KB
+#endif
+#ifndef TP_RING_SLACK_WORDS
+#define TP_RING_SLACK_WORDS 2048u          // the ring holds the largest item + 8 KB
 #endif
 #ifndef TP_STAR_RING_WORDS_GROUPED
 #define TP_STAR_RING_WORDS_GROUPED 6144u   // 24 KB
@@ -1023,9 +1047,6 @@ struct StarOp : OpBase {
   uint32_t* hhi;   // (a 64-bit shared atomicAdd is a CAS loop on sm_100)
   uint32_t* hcnt;
   uint32_t hmask, hshift;
-  // the held first measure: this thread's miniblock view (FOR) or row pointer (None)
-  const uint32_t* m1w;
-  uint32_t m1ref, m1b, m1none;
 
   __device__ void cta_init(const Params& P, uint32_t* smem) {
     if (GROUPED) {
@@ -1043,7 +1064,11 @@ struct StarOp : OpBase {
       }
     }
   }
+#if TP_HT_NOINLINE
+  __device__ __noinline__ void ht_add(uint32_t key, int64_t v) {
+#else
   __device__ __forceinline__ void ht_add(uint32_t key, int64_t v) {
+#endif
     uint32_t slot = (key * 0x9E3779B1u) >> hshift;  // multiplicative hash
 #pragma unroll 1
     for (uint32_t p = 0; p < HT_PROBES; ++p) {
@@ -1067,12 +1092,6 @@ struct StarOp : OpBase {
   }
   __device__ void begin(const Params& P, const StageCtx& C, const Lane& g) { alive = valid_rows(P, C, g); }
 
-  // the first measure of row i (the held item, or the staged array)
-  __device__ __forceinline__ uint32_t m1_at(uint32_t i, const uint32_t* W, uint32_t lane) const {
-    if (!A->hold_m1) return W[32u * i + lane];
-    if ((MASK & M_NONE) && m1none) return none_at(m1w, m1b, i);
-    return m1ref + extract_at(m1w, i * m1b, __funnelshift_lc(0xffffffffu, 0u, m1b));
-  }
   // the role of column c applied to row i (value x) -- shared by every mode
   __device__ __forceinline__ void apply_range(uint32_t c, uint32_t i, uint32_t x) {
     if ((uint32_t)((int32_t)x - A->lo[c]) > (uint32_t)(A->hi[c] - A->lo[c])) alive &= ~(1u << i);
@@ -1102,8 +1121,8 @@ struct StarOp : OpBase {
       for (int i = 0; i < 32; ++i) G[32u * i + lane] += p[i] * stride;
     }
   }
-  // measure role of row i: its own filter; the first measure is only filtered here (read back
-  // later), the aggregating one combines with it and aggregates
+  // measure role of row i: its own filter; the first measure is staged, the aggregating one
+  // combines with it and aggregates
   __device__ __forceinline__ void apply_measure(uint32_t c, uint32_t i, uint32_t x, const uint32_t* G, uint32_t* W,
                                                 uint32_t lane) {
     if ((uint32_t)((int32_t)x - A->lo[c]) > (uint32_t)(A->hi[c] - A->lo[c])) {
@@ -1111,12 +1130,12 @@ struct StarOp : OpBase {
       return;
     }
     if (A->mstage[c]) {
-      if (!A->hold_m1) W[32u * i + lane] = x;
+      W[32u * i + lane] = x;
       return;
     }
     int64_t y = (int32_t)x;
-    if (A->agg == TP_AGG_MUL) y *= (int64_t)(int32_t)m1_at(i, W, lane);
-    else if (A->agg == TP_AGG_SUB) y = (int64_t)(int32_t)m1_at(i, W, lane) - y;
+    if (A->agg == TP_AGG_MUL) y *= (int64_t)(int32_t)W[32u * i + lane];
+    else if (A->agg == TP_AGG_SUB) y = (int64_t)(int32_t)W[32u * i + lane] - y;
     if (GROUPED) ht_add(A->gzero ? 0u : G[32u * i + lane], y);
     else acc += (uint64_t)y;
   }
@@ -1195,7 +1214,7 @@ struct StarOp : OpBase {
   __device__ void rfor_col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c,
                            int role) {
     const Col& col = P.col[c];
-    const StreamView vv = stream_view(P, col.s0, C, 0), vl = stream_view(P, col.s1, C, 1);
+    const StreamView vv = stream_view<true>(P, col.s0, C, 0), vl = stream_view<true>(P, col.s1, C, 1);
     uint32_t* RA = scratch + A->ra_off;
     uint32_t* SB = scratch + A->sb_off;  // run-start bits per lane word
     uint32_t* PB = SB + 33;              // passing-run-start bits
@@ -1227,8 +1246,11 @@ struct StarOp : OpBase {
         tp_flag_error(4u);  // TP_DEVERR_RUNS
         r = 512u;
       }
-      if (r <= 128u) rfor_runs<4>(bV, bL, r, h, c, range, per_run, need_ra, all_alive, RA, SB, PB, AW, lane);
-      else rfor_runs<8>(bV, bL, r, h, c, range, per_run, need_ra, all_alive, RA, SB, PB, AW, lane);
+#if TP_RFOR_CC8
+      if (r > 128u) rfor_runs<8>(bV, bL, r, h, c, range, per_run, need_ra, all_alive, RA, SB, PB, AW, lane);
+      else
+#endif
+      rfor_runs<4>(bV, bL, r, h, c, range, per_run, need_ra, all_alive, RA, SB, PB, AW, lane);
     }
     __syncwarp();
     const uint32_t sb = SB[lane], jj = lane & 15u;
@@ -1275,27 +1297,9 @@ struct StarOp : OpBase {
     }
     const bool dfor = (MASK & M_DFOR) && col.scheme == S_DFOR;  // prefix sums: no random access
     const bool none = (MASK & M_NONE) && col.scheme == S_NONE;
-    const bool hold = A->hold_m1 && A->mstage[c];
     uint32_t* G = scratch + A->gs_off;
     uint32_t* W = scratch + A->ws_off;
     const uint32_t lane = g.lane;
-    if (hold) {  // this thread's view of the first measure, read back when the last column aggregates
-      if (none) {
-        uint32_t sw;
-        m1w = none_row(P, col, C, g, sw);
-        m1b = sw;
-        m1none = 1u;
-      } else {
-        const StreamView sv = stream_view(P, col.s0, C, 0);
-        uint32_t tl;
-        bool tv;
-        const MbView mv = for_mb(P, col, C, g, sv, tl, tv);
-        m1w = mv.w;
-        m1ref = mv.ref;
-        m1b = mv.b;
-        m1none = 0u;
-      }
-    }
     const uint32_t nal = __reduce_add_sync(FULL, __popc(alive));
     const bool sparse =
         !dfor && ((nal <= A->sparse_max &&
@@ -1307,7 +1311,7 @@ struct StarOp : OpBase {
     if (!sparse) {
       // ---------------- dense: every row of the warp's round
       uint32_t v[32];
-      decode_col<MASK & ~M_RFOR, TP_QUERY_COMPACT>(P, c, C, g, scratch, v);
+      decode_col<MASK & ~M_RFOR, TP_QUERY_COMPACT, true>(P, c, C, g, scratch, v);
       if (role == TP_ROLE_RANGE) {
 #pragma unroll
         for (int i = 0; i < 32; ++i) apply_range(c, i, v[i]);
@@ -1329,10 +1333,8 @@ struct StarOp : OpBase {
         for (int i = 0; i < 32; ++i)
           if ((uint32_t)((int32_t)v[i] - lo) > span) alive &= ~(1u << i);
         if (A->mstage[c]) {
-          if (!hold) {
 #pragma unroll
-            for (int i = 0; i < 32; ++i) W[32u * i + lane] = v[i];
-          }
+          for (int i = 0; i < 32; ++i) W[32u * i + lane] = v[i];
         } else {
           // (grouped: only a DFOR aggregating measure gets here, the others go sparse) -- static
           // row indices throughout: v[] stays in registers
@@ -1341,30 +1343,40 @@ struct StarOp : OpBase {
           for (int i = 0; i < 32; ++i) {
             if (m & (1u << i)) {
               int64_t y = (int32_t)v[i];
-              if (A->agg == TP_AGG_MUL) y *= (int64_t)(int32_t)m1_at(i, W, lane);
-              else if (A->agg == TP_AGG_SUB) y = (int64_t)(int32_t)m1_at(i, W, lane) - y;
+              if (A->agg == TP_AGG_MUL) y *= (int64_t)(int32_t)W[32u * i + lane];
+              else if (A->agg == TP_AGG_SUB) y = (int64_t)(int32_t)W[32u * i + lane] - y;
               if (GROUPED) ht_add(A->gzero ? 0u : G[32u * i + lane], y);
               else acc += (uint64_t)y;
             }
           }
         }
       }
-      return !hold;
+      return true;
     }
     // ---------------- sparse: alive rows only, values read out of the staged tile
     MbView mv;
     uint32_t bmask = 0u, nsw = 0u;
     const uint32_t* nw = nullptr;
     if (none) {
-      nw = none_row(P, col, C, g, nsw);
+      nw = none_row<true>(P, col, C, g, nsw);
     } else {
-      const StreamView sv = stream_view(P, col.s0, C, 0);
+      const StreamView sv = stream_view<true>(P, col.s0, C, 0);
       uint32_t tl;
       bool tv;
       mv = for_mb(P, col, C, g, sv, tl, tv);
       bmask = __funnelshift_lc(0xffffffffu, 0u, mv.b);
     }
     uint32_t m = alive;
+    if (role == TP_ROLE_MEASURE) {
+      // one row at a time (the aggregation's code once: instruction cache); few rows get here
+      while (m) {
+        const uint32_t i = __ffs(m) - 1u;
+        m &= m - 1u;
+        const uint32_t x = none ? none_at(nw, nsw, i) : mv.ref + extract_at(mv.w, i * mv.b, bmask);  // Alg. 1
+        apply_measure(c, i, x, G, W, lane);
+      }
+      return true;
+    }
     while (m) {
       uint32_t ii[4], xx[4];
       bool ok[4];
@@ -1379,7 +1391,7 @@ struct StarOp : OpBase {
 #pragma unroll
         for (int q = 0; q < 4; ++q)
           if (ok[q]) apply_range(c, ii[q], xx[q]);
-      } else if (role == TP_ROLE_PROBE) {
+      } else {
         const int32_t* __restrict__ T = A->table[c];
         const uint32_t kmin = (uint32_t)A->key_min[c], len = A->table_len[c];
         int32_t pl[4];
@@ -1391,13 +1403,9 @@ struct StarOp : OpBase {
 #pragma unroll
         for (int q = 0; q < 4; ++q)
           if (ok[q]) apply_payload(c, ii[q], pl[q], G, lane);
-      } else {
-#pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if (ok[q]) apply_measure(c, ii[q], xx[q], G, W, lane);
       }
     }
-    return !hold;
+    return true;
   }
   __device__ void end(const Params&, const StageCtx&, const Lane&) {
     if (!GROUPED) cnt += __popc(alive);
@@ -1469,8 +1477,6 @@ __global__ void __launch_bounds__(THREADS, GROUPED ? 3 : TP_STAR_MINB_UNGROUPED)
   op.acc = 0;
   op.cnt = 0;
   op.alive = 0;
-  op.m1w = nullptr;
-  op.m1ref = op.m1b = op.m1none = 0u;
   run_query_pipeline(P, op);
 }
 
@@ -1776,7 +1782,7 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
     P.ncols = (uint32_t)ncols;
     P.n = (uint32_t)n;
     P.ntiles = (uint32_t)((n + TILE_ROWS - 1) / TILE_ROWS);
-    P.ring_words = (std::max(ring_min_words, 2u * max_item) + 255u) & ~255u;
+    P.ring_words = (std::max(ring_min_words, max_item + TP_RING_SLACK_WORDS) + 255u) & ~255u;
     P.nstages = 0;
     P.stage_words = 0;
     P.staging_off = (any_rfor && rfor_scratch) ? RFOR_SCRATCH_WORDS : 0u;
@@ -1791,9 +1797,15 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
   // rounds per item: single-column kernels carry ~16 KB of compressed words per item
   // (bytes in flight at low bitwidths, where one round is a few hundred bytes); queries
   // keep per-round row state across columns, so they use one round per item
-  const uint32_t target_words = 4096;
+#ifndef TP_TARGET_WORDS
+#define TP_TARGET_WORDS 4096u  // ~16 KB of compressed words per single-column item
+#endif
+  const uint32_t target_words = TP_TARGET_WORDS;
   P.rounds = ncols > 1 ? 1u
                        : std::max<uint32_t>(1u, std::min<uint32_t>(8u, target_words / std::max(max_round_words, 1u)));
+#ifdef TP_FIXED_ROUNDS  // the tiles-per-item sweep (NEXT-4, Fig. 5): items of 8 x TP_FIXED_ROUNDS tiles
+  if (ncols == 1) P.rounds = TP_FIXED_ROUNDS;
+#endif
   const uint32_t TPS = TPR * P.rounds;
   uint32_t item = 0;
   for (int c = 0; c < ncols; ++c) {
@@ -1994,7 +2006,9 @@ tp_status tp_select_project_sum(const tp_column* dcols, int ncols, const int32_t
   }
   Params P;
   size_t smem = 0;
-  tp_status st = build_params(ord, k, 0, 0, P, smem, true, true, TP_STAR_RING_WORDS);
+  uint32_t ring_min = TP_STAR_RING_WORDS;
+  if (const char* e = getenv("TILEPACK_QUERY_RING_WORDS")) ring_min = (uint32_t)atoi(e);  // tests: a tight ring
+  tp_status st = build_params(ord, k, 0, 0, P, smem, true, true, ring_min);
   if (st != TP_OK) return st;
   auto out = reinterpret_cast<unsigned long long*>(d_result);
   const int cap = (int)((P.ntiles + 1) / 2);
@@ -2063,34 +2077,16 @@ tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int nc
   const uint32_t hts = grouped ? ht_slots(ngroups) : 0u;
   // byte ring: 24 KB next to the grouped queries' hash table and group arrays (3 CTAs / SM),
   // 32 KB for q1.x (4 CTAs / SM); at least twice the largest item either way
-  const uint32_t ring_min = grouped ? TP_STAR_RING_WORDS_GROUPED : TP_STAR_RING_WORDS;
+  uint32_t ring_min = grouped ? TP_STAR_RING_WORDS_GROUPED : TP_STAR_RING_WORDS;
+  if (const char* e = getenv("TILEPACK_QUERY_RING_WORDS")) ring_min = (uint32_t)atoi(e);  // tests: a tight ring
   bool any_rfor = false;
-  uint32_t mx = 0;
-  for (int c = 0; c < ncols; ++c) {
-    any_rfor |= dcols[c].scheme == TP_RFOR;
-    mx = std::max(mx, query_item_words(dcols[c]));
-  }
-  const uint32_t ring = (std::max(ring_min, 2u * mx) + 255u) & ~255u;
-  // the first measure stays in its ring item until the last column aggregates (no staging array)
-  // when it is random-access (FOR / None) and the items from it to the last column always fit
-  // in the ring next to one item of wrap-around waste
-  bool hold = false;
-  for (int c = 0; c < ncols - 1; ++c) {
-    if (roles[c].role != TP_ROLE_MEASURE) continue;
-    if (dcols[c].scheme == TP_FOR || dcols[c].scheme == TP_NONE) {
-      uint32_t span = 0;
-      for (int q = c; q < ncols; ++q) span += query_item_words(dcols[q]);
-      hold = span + mx <= ring;
-    }
-  }
-  if (const char* e = getenv("TILEPACK_STAR_NO_HOLD")) hold = hold && atoi(e) == 0;  // tests: the staged path
-  const uint32_t gwords = grouped ? 32u * 32u : 0u, wwords = nmeas == 2 && !hold ? 32u * 32u : 0u;
+  for (int c = 0; c < ncols; ++c) any_rfor |= dcols[c].scheme == TP_RFOR;
+  const uint32_t gwords = grouped ? 32u * 32u : 0u, wwords = nmeas == 2 ? 32u * 32u : 0u;
   const uint32_t rwords = any_rfor ? STAR_RA_WORDS + STAR_SB_WORDS : 0u;
   Params P;
   size_t smem = 0;
   tp_status st = build_params(dcols, ncols, gwords + wwords + rwords, 4u * hts, P, smem, true, false, ring_min);
   if (st != TP_OK) return st;
-  A.hold_m1 = hold ? 1u : 0u;
   A.gs_off = 0;
   A.ws_off = gwords;
   A.ra_off = gwords + wwords;

@@ -35,9 +35,10 @@ if __name__ == "__main__":
     if sys.argv[1] == "--child":
         child(int(sys.argv[2]))
         sys.exit(0)
-    libs = sys.argv[1:3]
-    bits = sys.argv[3] if len(sys.argv) > 3 else "16"
-    reps = int(sys.argv[4]) if len(sys.argv) > 4 else 3
+    libs = [a for a in sys.argv[1:] if a.endswith(".so")]
+    rest = [a for a in sys.argv[1:] if not a.endswith(".so")]
+    bits = rest[0] if rest else "16"
+    reps = int(rest[1]) if len(rest) > 1 else 3
     for r in range(reps):
         for lib in libs:
             env = dict(os.environ, TILEPACK_LIB_OVERRIDE=os.path.abspath(lib))

@@ -1,0 +1,91 @@
+#!/usr/bin/env python
+"""NEXT-4 (Fig. 5): the tiles-per-thread-block study on B200.  The paper sweeps D, the
+number of 128-value blocks a thread block decodes (D = 4: 1.55 ms at 500M U[0,2^16) on V100,
+P:954-956); here the corresponding knobs of the persistent TMA pipeline are swept for
+decode->sum at b = 4 and b = 16 (500M rows):
+  rounds  -- tiles per ring item = 8 x rounds (the single-column item; default: ~16 KB of words)
+  ring_kb -- the ring's bytes per CTA (default 40)
+  minb    -- CTAs per SM asked of the compiler (launch bounds; default 4)
+  python scripts/tile_sweep.py --build          (CPU: one library per point into build_ab/)
+  python scripts/tile_sweep.py --run OUT.json   (GPU: each library in its own process)"""
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+POINTS = {"default": ""}
+for r in (1, 2, 4, 8):
+    POINTS[f"rounds{r}"] = f"-DTP_FIXED_ROUNDS={r}"
+for kb in (16, 24, 64):
+    POINTS[f"ring{kb}kb"] = f"-DTP_RING_KB={kb}"
+for mb in (2, 3, 5):
+    POINTS[f"minb{mb}"] = f"-DTP_SUM_MINB={mb}"
+
+
+def build():
+    for name, flags in POINTS.items():
+        subprocess.check_call([sys.executable, os.path.join(ROOT, "scripts", "build_variant.py"), f"sw_{name}", flags],
+                              stdout=subprocess.DEVNULL)
+        print("built", name, flags, flush=True)
+
+
+def child(bits):
+    sys.path.insert(0, ROOT)
+    import numpy as np
+    import torch
+    import datagen
+    from paper_conf_sigmod_shanbhagyym22_b200 import tilepack as tp
+    x = datagen.uniform_bits(bits, 500_000_000, seed=2000 + bits)
+    h = tp.encode(x, "for")
+    d = h.to_device()
+    truth = int(x.astype(np.int64).sum())
+    acc = torch.zeros(1, dtype=torch.int64, device="cuda")
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+    for _ in range(3):
+        acc.zero_()
+        tp.tp_decode_sum(d.col, acc)
+    torch.cuda.synchronize()
+    ok = int(acc.item()) == truth
+    ts = []
+    for _ in range(15):
+        flush.zero_()
+        flush.sum()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        tp.tp_decode_sum(d.col, acc)
+        b.record()
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b))
+    sms, occ = tp.tp_device_info()
+    print("RESULT", json.dumps({"ms": float(np.median(ts)), "bytes": h.nbytes(), "parity": ok, "ctas_per_sm": occ}))
+
+
+def run(out):
+    peak = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"])
+    res = {"what": __doc__.split("\n\n")[0], "peak_hbm_gbs": peak, "points": {}}
+    for name, flags in POINTS.items():
+        lib = os.path.join(ROOT, "build_ab", f"libtilepack_sw_{name}.so")
+        for bits in (4, 16):
+            env = dict(os.environ, TILEPACK_LIB_OVERRIDE=lib)
+            o = subprocess.run([sys.executable, __file__, "--child", str(bits)], env=env, capture_output=True, text=True)
+            line = [x for x in o.stdout.splitlines() if x.startswith("RESULT")]
+            if not line:
+                print(name, bits, "FAILED", o.stderr[-500:], flush=True)
+                continue
+            r = json.loads(line[0][7:])
+            r["flags"] = flags
+            r["decoded_gbs"] = 2e9 / (r["ms"] / 1e3) / 1e9
+            r["hbm_frac"] = r["bytes"] / (r["ms"] / 1e3) / 1e9 / peak
+            res["points"][f"{name}_b{bits}"] = r
+            print(name, bits, json.dumps(r), flush=True)
+    json.dump(res, open(out, "w"), indent=1)
+
+
+if __name__ == "__main__":
+    if sys.argv[1] == "--build":
+        build()
+    elif sys.argv[1] == "--child":
+        child(int(sys.argv[2]))
+    else:
+        run(sys.argv[2])

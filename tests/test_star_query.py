@@ -71,10 +71,10 @@ def _cases(d):
         (["short", "long", "price"], ["rfor", "rfor", "for"],
          [dict(role="range", lo=0, hi=2000), dict(role="probe", table=d["t1"], key_min=0, stride=25), meas()],
          "sum", 7 * 25),
-        # RFOR range first, a held None first measure, a FOR probe, grouped difference
+        # RFOR range first, a None first measure, a FOR probe, grouped difference
         (["keys", "price", "fk", "cost"], ["rfor", "none", "for", "for"],
          [dict(role="range", lo=0, hi=1500), meas(), probe2, meas()], "sub", 25),
-        # ungrouped RFOR probe (filter only) on one-row runs, held FOR first measure, product
+        # ungrouped RFOR probe (filter only) on one-row runs, FOR first measure, product
         (["short", "cost", "price"], ["rfor", "for", "for"],
          [dict(role="probe", table=d["t1"], key_min=0, stride=0), meas(0, 90000), meas()], "mul", 1),
     ]
@@ -107,9 +107,8 @@ def test_oracle_star_query_brute_force():
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("hold", ["hold", "staged"])
 @pytest.mark.parametrize("mode", ["dense", "sparse", "auto"])
-def test_gpu_star_query_modes(mode, hold, monkeypatch):
+def test_gpu_star_query_modes(mode, monkeypatch):
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
@@ -117,19 +116,21 @@ def test_gpu_star_query_modes(mode, hold, monkeypatch):
     if mode != "auto":
         monkeypatch.setenv("TILEPACK_SPARSE_MAX", "0" if mode == "dense" else "1024")
         monkeypatch.setenv("TILEPACK_SPARSE_LANE_MAX", "0" if mode == "dense" else "32")
-    if hold == "staged":  # the first measure staged per row instead of read back from its ring item
-        monkeypatch.setenv("TILEPACK_STAR_NO_HOLD", "1")
     _run_cases(torch, tp, N, (1, 2), mode)
 
 
 @pytest.mark.gpu
-def test_gpu_star_query_long_columns():
+@pytest.mark.parametrize("ring", ["default", "tight"])
+def test_gpu_star_query_long_columns(ring, monkeypatch):
     """20M rows: every CTA runs tens of rounds, so the byte ring wraps many times with items of
-    very different sizes (RFOR 6-bit keys next to 25-bit FOR prices) and held first measures."""
+    very different sizes (RFOR 6-bit keys next to 25-bit FOR prices);
+    'tight': the smallest ring the host allows (the largest item + the slack)."""
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
     from paper_conf_sigmod_shanbhagyym22_b200 import tilepack as tp
+    if ring == "tight":
+        monkeypatch.setenv("TILEPACK_QUERY_RING_WORDS", "0")
     _run_cases(torch, tp, 20_000_000 + 333, (3,), "auto")
     assert tp.tp_device_errors() == 0
 
