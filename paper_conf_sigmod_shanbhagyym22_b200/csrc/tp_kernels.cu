@@ -578,6 +578,9 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
 // column held two items of an SSB query).  An operator may keep an item until the end of its
 // round (Op::col returns false); the host must then size the ring for every item in between.
 constexpr uint32_t QNS = 16;
+#ifndef TP_QUERY_PREFETCH
+#define TP_QUERY_PREFETCH 2  // rounds the query producer prefetches into L2 ahead of the ring
+#endif
 #ifndef TP_QPROD_SPIN
 #define TP_QPROD_SPIN 0
 #endif
@@ -627,6 +630,26 @@ __device__ __forceinline__ void run_query_pipeline(const Params& P, Op& op) {
       const uint32_t ge = min(gb + 31, ngr);
       for (uint32_t g = gb; g < ge; ++g) {
         const uint32_t tile_base = t0 + g * TPR, tile_end = min(tile_base + TPR, t1);
+#if TP_QUERY_PREFETCH
+        // the ring holds about one round of a multi-column query: run TP_QUERY_PREFETCH rounds
+        // ahead in L2 (bulk prefetches of every stream's words), so that the ring's TMA copies
+        // are served from L2 rather than HBM (measured: consumers spun on data 15-20 % of their
+        // instructions without it)
+        if (g + TP_QUERY_PREFETCH < ge) {
+          const uint32_t rel = g + TP_QUERY_PREFETCH - gb;
+#pragma unroll
+          for (int q = 0; q < MAX_STREAMS; ++q) {
+            if ((uint32_t)q < P.nstreams) {
+              const uint32_t a = __shfl_sync(FULL, bnd[q], rel), b = __shfl_sync(FULL, bnd[q], rel + 1);
+              if (lane == (uint32_t)q && b > a) {
+                const uintptr_t a0 = reinterpret_cast<uintptr_t>(P.st[q].data + a) & ~uintptr_t(15);
+                const uintptr_t a1 = (reinterpret_cast<uintptr_t>(P.st[q].data + b) + 15) & ~uintptr_t(15);
+                bulk_prefetch_l2(reinterpret_cast<const void*>(a0), (uint32_t)(a1 - a0));
+              }
+            }
+          }
+        }
+#endif
         for (uint32_t c = 0; c < P.ncols; ++c, ++item) {
           const Col& cc = P.col[c];
           const uint32_t my_s = lane == 0 ? cc.s0 : (lane == 1 && cc.scheme == S_RFOR ? cc.s1 : 0xffu);
@@ -676,6 +699,9 @@ __device__ __forceinline__ void run_query_pipeline(const Params& P, Op& op) {
           uint32_t hd = none ? (head + 255u) & ~255u : head;
           if (hd % RW + need > RW) hd += RW - hd % RW;  // does not fit before the ring's end: wrap
           // reclaim: the slot's previous item, and every item still holding the space needed
+#ifdef TP_PROFILE_WAITS
+          const long long pw0 = clock64();
+#endif
           while (item - oldest >= QNS || (oldest < item && hd + need > __shfl_sync(FULL, vst, oldest % QNS) + RW)) {
 #if TP_QPROD_SPIN
             mbar_wait(&empty[oldest % QNS], (oldest / QNS) & 1u);
@@ -684,6 +710,9 @@ __device__ __forceinline__ void run_query_pipeline(const Params& P, Op& op) {
 #endif
             ++oldest;
           }
+#ifdef TP_PROFILE_WAITS
+          if (lane == 0) atomicAdd(&g_prof[8], (unsigned long long)(clock64() - pw0));
+#endif
           const uint32_t slot = item % QNS;
           if (lane == slot) vst = hd;
           head = hd + need;
@@ -718,12 +747,24 @@ __device__ __forceinline__ void run_query_pipeline(const Params& P, Op& op) {
       uint32_t held = 0xffffffffu;
       for (uint32_t c = 0; c < P.ncols; ++c, ++item) {
         const uint32_t slot = item % QNS;
+#ifdef TP_PROFILE_WAITS
+        const long long w0 = clock64();
+#endif
         mbar_wait_backoff(&full[slot], (item / QNS) & 1u);
+#ifdef TP_PROFILE_WAITS
+        const long long w1 = clock64();
+#endif
         const uint4 mt = *reinterpret_cast<const uint4*>(meta + 4u * slot);
         C.stage = smem + mt.x;
         C.doff[0] = 0u; C.soff[0] = mt.y; C.doff[1] = mt.z; C.soff[1] = mt.w;
         const bool rel = op.col(P, C, g, scratch, c, gi);
         __syncwarp();
+#ifdef TP_PROFILE_WAITS
+        if (g.lane == 0) {
+          atomicAdd(&g_prof[0], (unsigned long long)(w1 - w0));
+          atomicAdd(&g_prof[1 + min(c, 6u)], (unsigned long long)(clock64() - w1));
+        }
+#endif
         if (rel) {
           if (g.lane == 0) mbar_arrive(&empty[slot]);
         } else {
@@ -1798,7 +1839,8 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
   // (bytes in flight at low bitwidths, where one round is a few hundred bytes); queries
   // keep per-round row state across columns, so they use one round per item
 #ifndef TP_TARGET_WORDS
-#define TP_TARGET_WORDS 4096u  // ~16 KB of compressed words per single-column item
+#define TP_TARGET_WORDS 8192u  // ~32 KB of compressed words per single-column item (NEXT-4 sweep:
+                               // b = 16 0.169 -> 0.159 ms vs 16 KB items, profiles/r02_tile_sweep*.json)
 #endif
   const uint32_t target_words = TP_TARGET_WORDS;
   P.rounds = ncols > 1 ? 1u

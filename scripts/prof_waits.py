@@ -16,7 +16,7 @@ def main():
     import datagen.ssb as gen
     from paper_conf_sigmod_shanbhagyym22_b200 import tilepack as tp
     from paper_conf_sigmod_shanbhagyym22_b200.ssb import SSBEngine
-    eng = SSBEngine(gen.generate(sf, seed=5000, columns=gen.QUERY_COLUMNS))
+    eng = SSBEngine(gen.generate(sf, seed=5000, columns=gen.QUERY_COLUMNS))  # noqa
     for q in qs:
         prep = eng.prepare(q)
         eng.execute(prep)

@@ -21,23 +21,37 @@ for kb in (16, 24, 64):
     POINTS[f"ring{kb}kb"] = f"-DTP_RING_KB={kb}"
 for mb in (2, 3, 5):
     POINTS[f"minb{mb}"] = f"-DTP_SUM_MINB={mb}"
+# second sweep: the item-size target and the ring of the instruction-bound single-column decodes
+POINTS2 = {"default": ""}
+for tw in (6144, 8192, 12288):
+    POINTS2[f"tw{tw}"] = f"-DTP_TARGET_WORDS={tw}u"
+for kb in (40, 64):
+    POINTS2[f"qring{kb}kb"] = f"-DTP_QUERY_RING_KB={kb}"
+POINTS2["tw8192_qring40kb"] = "-DTP_TARGET_WORDS=8192u -DTP_QUERY_RING_KB=40"
+CONFIGS = {"for_b4": ("for", lambda n: __import__("datagen").uniform_bits(4, n, seed=2004)),
+           "for_b16": ("for", lambda n: __import__("datagen").uniform_bits(16, n, seed=2016)),
+           "dfor_d1": ("dfor", lambda n: __import__("datagen").d1_sorted(n, 2**28)),
+           "rfor_runs8": ("rfor", lambda n: __import__("datagen").runs(n, 8))}
 
 
-def build():
-    for name, flags in POINTS.items():
+def build(points=POINTS):
+    for name, flags in points.items():
         subprocess.check_call([sys.executable, os.path.join(ROOT, "scripts", "build_variant.py"), f"sw_{name}", flags],
                               stdout=subprocess.DEVNULL)
         print("built", name, flags, flush=True)
 
 
-def child(bits):
+def child(cfg):
     sys.path.insert(0, ROOT)
     import numpy as np
     import torch
-    import datagen
     from paper_conf_sigmod_shanbhagyym22_b200 import tilepack as tp
-    x = datagen.uniform_bits(bits, 500_000_000, seed=2000 + bits)
-    h = tp.encode(x, "for")
+    if cfg.isdigit():
+        scheme, gen = "for", (lambda n: __import__("datagen").uniform_bits(int(cfg), n, seed=2000 + int(cfg)))
+    else:
+        scheme, gen = CONFIGS[cfg]
+    x = gen(500_000_000)
+    h = tp.encode(x, scheme)
     d = h.to_device()
     truth = int(x.astype(np.int64).sum())
     acc = torch.zeros(1, dtype=torch.int64, device="cuda")
@@ -61,12 +75,12 @@ def child(bits):
     print("RESULT", json.dumps({"ms": float(np.median(ts)), "bytes": h.nbytes(), "parity": ok, "ctas_per_sm": occ}))
 
 
-def run(out):
+def run(out, points=POINTS, cfgs=("4", "16"), prefix="sw_"):
     peak = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"])
     res = {"what": __doc__.split("\n\n")[0], "peak_hbm_gbs": peak, "points": {}}
-    for name, flags in POINTS.items():
-        lib = os.path.join(ROOT, "build_ab", f"libtilepack_sw_{name}.so")
-        for bits in (4, 16):
+    for name, flags in points.items():
+        lib = os.path.join(ROOT, "build_ab", f"libtilepack_{prefix}{name}.so")
+        for bits in cfgs:
             env = dict(os.environ, TILEPACK_LIB_OVERRIDE=lib)
             o = subprocess.run([sys.executable, __file__, "--child", str(bits)], env=env, capture_output=True, text=True)
             line = [x for x in o.stdout.splitlines() if x.startswith("RESULT")]
@@ -77,7 +91,7 @@ def run(out):
             r["flags"] = flags
             r["decoded_gbs"] = 2e9 / (r["ms"] / 1e3) / 1e9
             r["hbm_frac"] = r["bytes"] / (r["ms"] / 1e3) / 1e9 / peak
-            res["points"][f"{name}_b{bits}"] = r
+            res["points"][f"{name}_{'b' + bits if bits.isdigit() else bits}"] = r
             print(name, bits, json.dumps(r), flush=True)
     json.dump(res, open(out, "w"), indent=1)
 
@@ -85,7 +99,11 @@ def run(out):
 if __name__ == "__main__":
     if sys.argv[1] == "--build":
         build()
+    elif sys.argv[1] == "--build2":
+        build({f"sw2_{k}": v for k, v in POINTS2.items()})
     elif sys.argv[1] == "--child":
-        child(int(sys.argv[2]))
+        child(sys.argv[2])
+    elif sys.argv[1] == "--run2":
+        run(sys.argv[2], POINTS2, ("for_b4", "for_b16", "dfor_d1", "rfor_runs8"), "sw2_")
     else:
         run(sys.argv[2])
