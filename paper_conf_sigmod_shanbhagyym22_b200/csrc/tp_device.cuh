@@ -246,12 +246,16 @@ __device__ __forceinline__ void unpack_any(const uint32_t* __restrict__ w, uint3
 #define TP_UNPACK_MAX_PASSES 2
 #endif
 __device__ __forceinline__ void unpack_mb(const uint32_t* __restrict__ w, uint32_t b, uint32_t (&e)[32]) {
-  const uint32_t zl = __ballot_sync(FULL, b == 0u);
-  uint32_t todo = zl == FULL ? FULL : ~zl;  // the non-empty lanes (or all of them, if all empty)
+  const uint32_t bmin = __reduce_min_sync(FULL, b), bmax = __reduce_max_sync(FULL, b);
+  const bool uniform = bmin == bmax;  // one width across the warp (the common case): one pass
+  uint32_t todo = FULL, ride = 0u, zl = 0u;
+  if (!uniform) {
+    zl = __ballot_sync(FULL, b == 0u);
+    todo = zl == FULL ? FULL : ~zl;  // the non-empty lanes (or all of them, if all empty)
+    ride = zl == FULL ? 0u : zl;     // empty lanes joining the first pass
 #if TP_UNPACK_MAX_PASSES < 32
-  // more distinct bitwidths than TP_UNPACK_MAX_PASSES among the lanes (delta streams of
-  // near-sorted keys): one runtime-bitwidth pass beats several specialised ones
-  {
+    // more distinct bitwidths than TP_UNPACK_MAX_PASSES among the lanes (delta streams of
+    // near-sorted keys): one runtime-bitwidth pass beats several specialised ones
     uint32_t t = todo;
 #pragma unroll
     for (int k = 0; k < TP_UNPACK_MAX_PASSES; ++k) {
@@ -263,11 +267,10 @@ __device__ __forceinline__ void unpack_mb(const uint32_t* __restrict__ w, uint32
       unpack_any(w, b, e);
       return;
     }
-  }
 #endif
-  uint32_t ride = zl == FULL ? 0u : zl;  // empty lanes joining the first pass
+  }
   do {
-    const uint32_t bl = __shfl_sync(FULL, b, __ffs(todo) - 1);
+    const uint32_t bl = uniform ? bmin : __shfl_sync(FULL, b, __ffs(todo) - 1);
     const bool mine = b == bl || ((ride >> (threadIdx.x & 31u)) & 1u);
     todo &= ~__ballot_sync(FULL, b == bl);
     ride = 0u;

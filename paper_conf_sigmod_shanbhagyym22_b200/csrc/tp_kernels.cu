@@ -789,6 +789,9 @@ __device__ __forceinline__ void consumers_sync() {
 #ifndef TP_SPARSE_LANE_MAX
 #define TP_SPARSE_LANE_MAX 8  // ... and (FOR filters / measures) the busiest lane's alive rows
 #endif
+#ifndef TP_RFOR_SPARSE_MAX
+#define TP_RFOR_SPARSE_MAX 32  // (<= 32: one alive row per lane)
+#endif
 #ifndef TP_SPARSE_MAX
 #define TP_SPARSE_MAX 512  // alive rows (of a warp's 1024) at or below which a column goes sparse
                            // (512 / 8 measured best over the 13 SSB queries at SF20)
@@ -1045,6 +1048,8 @@ struct StarArgs {
   uint32_t sparse_max;           // warp alive-row count at or below which a column is evaluated sparsely
   uint32_t sparse_lane_max;      // ... and the busiest lane's alive rows: the sparse loop runs for the
                                  // warp's maximum (alive rows cluster: runs of an order's lines)
+  uint32_t rfor_sparse_max;      // a GPU-RFOR column with at most this many alive rows (<= 32) in the
+                                 // warp goes sparse (run lengths only + a binary search per row)
   long long* sums;
   unsigned long long* counts;
 };
@@ -1252,6 +1257,120 @@ struct StarOp : OpBase {
       }
     }
   }
+  // sparse GPU-RFOR (few alive rows): only the run-length stream is unpacked -- its scan gives
+  // every run's start row (Sarr[e], e < r) -- and each alive row finds its run by binary search
+  // and unpacks that one run value (random access into the value stream block, Alg. 1 for one
+  // entry); the alive rows are spread one per lane (compaction), so the warp runs one pass for
+  // up to 32 rows whatever their owner lanes
+  __device__ __forceinline__ void rfor_starts(const uint32_t* bL, uint32_t r, uint32_t lane, uint32_t* Sarr) {
+    const uint32_t refL = bL[1];
+    const uint4 wl = make_uint4(bL[2], bL[3], bL[4], bL[5]);
+    uint32_t rows = 0u;
+#pragma unroll 1
+    for (uint32_t e00 = 0; e00 < r; e00 += 128u) {
+      const uint32_t e0 = e00 + 4u * lane, m = (e0 >> 5) & 15u, pos = e0 & 31u;
+      const uint32_t bl = checked_bw(byte_of(wl, m));
+      const uint32_t* mL = bL + 6 + bytes_before(wl, m);
+      const uint32_t ml = __funnelshift_lc(0xffffffffu, 0u, bl);
+      uint32_t len[4], run = 0u;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        len[k] = e0 + k < r ? refL + extract_at(mL, (pos + k) * bl, ml) : 0u;
+        run += len[k];
+      }
+      const uint32_t incl = warp_inclusive_scan(run, lane);
+      uint32_t S = rows + incl - run;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        if (e0 + k < r) Sarr[e0 + k] = S;
+        S += len[k];
+      }
+      rows += __shfl_sync(FULL, incl, 31);
+    }
+  }
+  __device__ void rfor_col_sparse(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c,
+                                  int role, uint32_t nal) {
+    const Col& col = P.col[c];
+    const StreamView vv = stream_view<true>(P, col.s0, C, 0), vl = stream_view<true>(P, col.s1, C, 1);
+    uint32_t* RA = scratch + A->ra_off;  // run starts of both blocks (block h at 512 h)
+    uint32_t* LS = scratch + A->sb_off;  // the warp's alive rows, compacted (<= 32)
+    uint32_t* AW = LS + 66;              // alive words
+    uint32_t* G = scratch + A->gs_off;
+    uint32_t* W = scratch + A->ws_off;
+    const uint32_t lane = g.lane;
+    __syncwarp();  // the previous RFOR column's readers are done
+    {
+      const uint32_t cnt = __popc(alive);
+      uint32_t off = warp_inclusive_scan(cnt, lane) - cnt, m = alive;
+      while (m) {
+        const uint32_t i = __ffs(m) - 1u;
+        m &= m - 1u;
+        LS[off++] = (lane << 5) | i;
+      }
+      AW[lane] = alive;
+    }
+    const uint32_t live_lanes = __ballot_sync(FULL, alive != 0u);
+    const uint32_t* bV0 = nullptr;
+    const uint32_t* bV1 = nullptr;
+    uint32_t r0 = 0u, r1 = 0u;
+#pragma unroll
+    for (uint32_t h = 0; h < 2; ++h) {
+      const uint32_t tl = C.round_base + 2u * g.cw + h;
+      if (C.t0s + tl >= C.tile_end) break;                          // warp-uniform
+      if (((live_lanes >> (16u * h)) & 0xffffu) == 0u) continue;  // no alive row in this block
+      const uint32_t* bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
+      const uint32_t* bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
+      uint32_t r = bL[0];
+      if (r > 512u) {
+        tp_flag_error(4u);  // TP_DEVERR_RUNS
+        r = 512u;
+      }
+      if (h == 0) { bV0 = bV; r0 = r; } else { bV1 = bV; r1 = r; }
+      rfor_starts(bL, r, lane, RA + 512u * h);
+    }
+    __syncwarp();
+    if (lane < nal) {
+      const uint32_t id = LS[lane], j = id >> 5, i = id & 31u, h = j >> 4;
+      const uint32_t q = 32u * (j & 15u) + i;  // the row within its block
+      const uint32_t* Sa = RA + 512u * h;
+      uint32_t lo = 0u, hi = h ? r1 : r0;  // the last run starting at or before q (row 0 starts run 0)
+      while (hi - lo > 1u) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (Sa[mid] <= q) lo = mid; else hi = mid;
+      }
+      const uint32_t* bV = h ? bV1 : bV0;
+      const uint4 wv = make_uint4(bV[2], bV[3], bV[4], bV[5]);
+      const uint32_t mb = lo >> 5, bv = checked_bw(byte_of(wv, mb));
+      const uint32_t x = bV[1] + extract_at(bV + 6 + bytes_before(wv, mb), (lo & 31u) * bv,
+                                            __funnelshift_lc(0xffffffffu, 0u, bv));  // the run's value
+      bool kill = false;
+      if (role == TP_ROLE_RANGE) {
+        kill = (uint32_t)((int32_t)x - A->lo[c]) > (uint32_t)(A->hi[c] - A->lo[c]);
+      } else if (role == TP_ROLE_PROBE) {
+        const uint32_t kk = x - (uint32_t)A->key_min[c];
+        const int32_t p = kk < A->table_len[c] ? __ldg(A->table[c] + kk) : -1;
+        kill = p < 0;
+        if (!kill && GROUPED && A->gmode[c]) {
+          uint32_t* gp = G + 32u * i + j;
+          *gp = (A->gmode[c] == 1 ? 0u : *gp) + (uint32_t)p * A->stride[c];
+        }
+      } else if ((uint32_t)((int32_t)x - A->lo[c]) > (uint32_t)(A->hi[c] - A->lo[c])) {
+        kill = true;  // the measure's own filter
+      } else if (A->mstage[c]) {
+        W[32u * i + j] = x;
+      } else {
+        int64_t y = (int32_t)x;
+        if (A->agg == TP_AGG_MUL) y *= (int64_t)(int32_t)W[32u * i + j];
+        else if (A->agg == TP_AGG_SUB) y = (int64_t)(int32_t)W[32u * i + j] - y;
+        if (GROUPED) ht_add(A->gzero ? 0u : G[32u * i + j], y);
+        else acc += (uint64_t)y;
+      }
+      if (kill) atomicAnd(&AW[j], ~(1u << i));
+    }
+    __syncwarp();
+    alive = AW[lane];
+  }
+
   __device__ void rfor_col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t c,
                            int role) {
     const Col& col = P.col[c];
@@ -1333,7 +1452,9 @@ struct StarOp : OpBase {
     const int role = A->role[c];
     const Col& col = P.col[c];
     if ((MASK & M_RFOR) && col.scheme == S_RFOR) {
-      rfor_col(P, C, g, scratch, c, role);
+      const uint32_t nal = __reduce_add_sync(FULL, __popc(alive));
+      if (nal <= A->rfor_sparse_max) rfor_col_sparse(P, C, g, scratch, c, role, nal);
+      else rfor_col(P, C, g, scratch, c, role);
       return true;
     }
     const bool dfor = (MASK & M_DFOR) && col.scheme == S_DFOR;  // prefix sums: no random access
@@ -2114,6 +2235,8 @@ tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int nc
   A.ngroups = ngroups;
   A.sparse_max = TP_SPARSE_MAX;
   A.sparse_lane_max = TP_SPARSE_LANE_MAX;
+  A.rfor_sparse_max = TP_RFOR_SPARSE_MAX;
+  if (const char* e = getenv("TILEPACK_RFOR_SPARSE_MAX")) A.rfor_sparse_max = std::min(32, atoi(e));  // tests
   if (const char* e = getenv("TILEPACK_SPARSE_LANE_MAX")) A.sparse_lane_max = (uint32_t)atoi(e);  // tuning
   if (const char* e = getenv("TILEPACK_SPARSE_MAX")) A.sparse_max = (uint32_t)atoi(e);  // tests: force a mode
   const uint32_t hts = grouped ? ht_slots(ngroups) : 0u;

@@ -77,6 +77,15 @@ def _cases(d):
         # ungrouped RFOR probe (filter only) on one-row runs, FOR first measure, product
         (["short", "cost", "price"], ["rfor", "for", "for"],
          [dict(role="probe", table=d["t1"], key_min=0, stride=0), meas(0, 90000), meas()], "mul", 1),
+        # a selective FOR filter first (~20 of a warp's 1024 rows), then RFOR columns in every role
+        # with few alive rows (the sparse RFOR path: run lengths + a binary search per row):
+        # a grouped payload probe, a range, an RFOR first measure and an RFOR aggregating one
+        (["qty", "keys", "short", "long", "keys"], ["for", "rfor", "rfor", "rfor", "rfor"],
+         [dict(role="range", lo=7, hi=7), probe1, dict(role="range", lo=0, hi=2500), meas(), meas(0, 2900)],
+         "sub", 7 * 25),
+        (["qty", "long", "keys"], ["for", "rfor", "rfor"],
+         [dict(role="range", lo=3, hi=3), dict(role="probe", table=d["t1"], key_min=0, stride=0), meas()],
+         "sum", 1),
     ]
 
 
@@ -116,6 +125,7 @@ def test_gpu_star_query_modes(mode, monkeypatch):
     if mode != "auto":
         monkeypatch.setenv("TILEPACK_SPARSE_MAX", "0" if mode == "dense" else "1024")
         monkeypatch.setenv("TILEPACK_SPARSE_LANE_MAX", "0" if mode == "dense" else "32")
+        monkeypatch.setenv("TILEPACK_RFOR_SPARSE_MAX", "0" if mode == "dense" else "32")
     _run_cases(torch, tp, N, (1, 2), mode)
 
 
