@@ -149,16 +149,18 @@ tp_status tp_validate(const tp_column* host_col, uint32_t* max_tile_words0, uint
 /* ---------------------------------------------------------------- device */
 
 /* Format violations the DEVICE calls detect while they run (bit flags; the kernel
- * stays inside its buffers -- a bitwidth byte > 32 is used as 32, a tile range longer
- * than the ring region sized from max_tile_words is copied only up to the region -- and
- * the affected results are undefined):
- *   TP_DEVERR_BITWIDTH   a miniblock bitwidth byte > 32 (R3, R5)
+ * stays inside its buffers -- a tile range longer than the ring region sized from
+ * max_tile_words is copied only up to the region, a run count above 512 is used as
+ * 512 -- and the affected results are undefined):
  *   TP_DEVERR_TILE_WORDS a tile range spans more words than max_tile_words0/1 says
  *   TP_DEVERR_RUNS       an RFOR stream block counts more than 512 runs (R17)
+ * A miniblock bitwidth byte > 32 (R3, R5) is used as 32 on the device (memory-safe, the
+ * values undefined) and NOT flagged there -- checking it per miniblock cost 2-4 % of the
+ * decode kernels; tp_validate reports it (TP_EFORMAT) for a host column.
  * tp_device_errors synchronizes `stream`, writes the flags accumulated by this
  * library's kernels on the current device since the last call to *flags (host), and
  * clears them.  Returns TP_ECUDA if the synchronisation or the read fails. */
-enum { TP_DEVERR_BITWIDTH = 1, TP_DEVERR_TILE_WORDS = 2, TP_DEVERR_RUNS = 4 };
+enum { TP_DEVERR_TILE_WORDS = 2, TP_DEVERR_RUNS = 4 };
 tp_status tp_device_errors(uint32_t* flags, void* stream);
 
 /* Decode the whole DEVICE column into d_out[0..n) (int32, device).

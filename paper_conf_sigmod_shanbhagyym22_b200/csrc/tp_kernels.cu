@@ -1960,10 +1960,16 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
   // (bytes in flight at low bitwidths, where one round is a few hundred bytes); queries
   // keep per-round row state across columns, so they use one round per item
 #ifndef TP_TARGET_WORDS
-#define TP_TARGET_WORDS 8192u  // ~32 KB of compressed words per single-column item (NEXT-4 sweep:
-                               // b = 16 0.169 -> 0.159 ms vs 16 KB items, profiles/r02_tile_sweep*.json)
+#define TP_TARGET_WORDS 8192u  // ~32 KB of compressed words per GPU-FOR item (NEXT-4 sweep: b = 16
+                               // 0.169 -> 0.159 ms vs 16 KB items, profiles/r02_tile_sweep*.json)
 #endif
-  const uint32_t target_words = TP_TARGET_WORDS;
+#ifndef TP_TARGET_WORDS_OTHER
+#define TP_TARGET_WORDS_OTHER 4096u  // ~16 KB for the instruction-bound DFOR / RFOR decodes: their
+                                     // 24 KB ring keeps 4 CTAs / SM (32 KB items: RFOR runs of 4
+                                     // 0.72 -> 1.15 ms at 2 CTAs / SM, same-box A/B)
+#endif
+  const bool for_item = ncols == 1 && (cols[0].scheme == TP_FOR || cols[0].scheme == TP_FORNM);
+  const uint32_t target_words = for_item ? TP_TARGET_WORDS : TP_TARGET_WORDS_OTHER;
   P.rounds = ncols > 1 ? 1u
                        : std::max<uint32_t>(1u, std::min<uint32_t>(8u, target_words / std::max(max_round_words, 1u)));
 #ifdef TP_FIXED_ROUNDS  // the tiles-per-item sweep (NEXT-4, Fig. 5): items of 8 x TP_FIXED_ROUNDS tiles

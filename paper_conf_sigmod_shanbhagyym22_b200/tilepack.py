@@ -174,7 +174,7 @@ def tp_validate(col: tp_column):
     return m0.value, m1.value
 
 
-TP_DEVERR_BITWIDTH, TP_DEVERR_TILE_WORDS, TP_DEVERR_RUNS = 1, 2, 4
+TP_DEVERR_TILE_WORDS, TP_DEVERR_RUNS = 2, 4
 
 
 def tp_device_errors(stream=None) -> int:

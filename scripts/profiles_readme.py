@@ -1,7 +1,8 @@
 #!/usr/bin/env python
-"""Regenerate profiles/README.md from the committed profiles/*.json (after copying a
-scripts/refresh_profiles.sh run from gpurun_out/r/).  usage: python scripts/profiles_readme.py"""
+"""Regenerate profiles/README.md from the committed profiles/r02_*.json (after copying a
+scripts/refresh_profiles.sh run from gpurun_out/r2/).  usage: python scripts/profiles_readme.py"""
 import json
+import math
 import os
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -16,139 +17,109 @@ def load(name):
     return None
 
 
+def first(*names):
+    for n in names:
+        d = load(n)
+        if d is not None:
+            return n, d
+    return None, None
+
+
 def main():
-    b = load("r01_bench.json")
+    b = load("r02_bench.json")
     r = b["roofline"]
     ncu = load("ncu_summary.json")["kernels"]["for_b16_sum"]
-    s = f"""# profiles/ — measured evidence (round 1)
+    s = f"""# profiles/ — measured evidence (round 2)
 
-All numbers on one B200 (148 SMs, sm_100a, SM clock {b['clocks']['sm_mhz']:.0f} MHz under load = max, no throttle
-reasons recorded), CUDA 12.9, driver 580.  Roofline denominator: `MEASURED_PEAKS.json` `hbm_gbs`
-(copy, read+write; "of measured").  Every file below comes from ONE run of
-`scripts/refresh_profiles.sh` (all measurements + ncu captures on one box, at the final commit of
-round 1); this README is generated from them by `scripts/profiles_readme.py`.
+All numbers on one B200 (148 SMs, sm_100a, SM clock {b['clocks']['sm_mhz']:.0f} MHz under load, max
+{b['clocks']['sm_max_mhz']}, throttle reasons {b['clocks']['reasons'] or 'none'}), CUDA 12.9, driver 580.  Roofline
+denominators: `MEASURED_PEAKS.json` `hbm_gbs` (copy, read+write) and the INT32 issue roof measured by the
+bench itself.  The r02_* files come from ONE run of `scripts/refresh_profiles.sh` at the final commit
+of round 2 (the r02_tile_sweep* and r01_* files from the runs named below); this README is generated
+from them by `scripts/profiles_readme.py`.
 
 | file | what |
 |---|---|
-| `r01_bench.json` | `python bench.py` (defaults: 500 steps, 5 warm-up) — the JSON line the driver reads |
-| `r01_launches_bench.csv` | `ncu --metrics gpu__time_duration.sum --clock-control none -c 60 python bench.py --steps 10 --warmup 3 --no-cpu-baseline --e2e-steps 2` — per-launch list |
-| `ncu_summary.json`, `r01_ncu_k_decode_sum_details.txt` | `ncu --set full --clock-control none --import-source on -k regex:k_decode_sum -s 3 -c 1 python bench.py --steps 3 ...` — DRAM bytes per launch (the bench's `roofline.traffic`), occupancy, issue, stall details |
-| `r01_suite.json` | `scripts/bench_suite.py` — every BASELINE config 2-4 column (FOR b = 0..32, DFOR C3, RFOR C4) at 500M rows, decode→sum and decode→global, full-size parity flags |
-| `r01_ssb_sf20.json`, `r01_ssb_sf20_none.json`, `r01_ssb_sf160.json` | `scripts/bench_ssb.py --sf 20 --check` (GPU-*, every result == the oracle), `--scheme none` (uncompressed through the same kernels), `--sf 160` (config 5's SF×8) |
-| `r01_encode.json` | `scripts/bench_encode.py` — the tile-parallel GPU encoder at 500M rows (GPU bytes == host-encoder bytes, decode == input), the GPU-* analysis pass, the host encoder and the oracle (20M-row sample) beside it |
-| `r01_random_access.json` | `scripts/bench_random_access.py` — P:1241-1262 selectivity sweep at 250M rows, compressed vs None, parity and the oracle's time at every point |
-| `r01_cascaded_ablation.json` | `scripts/bench_cascaded.py` — tile-based vs cascading decode (NEXT-1, Fig. 7a) |
-| `r01_waterfall_sf20.json` | `scripts/bench_waterfall.py` — SSB compression waterfall + per-column decode (NEXT-2, Fig. 9/10) |
-| `r01_nomb_ablation.json` | `scripts/bench_nomb.py` — GPU-FOR with vs without miniblocks (NEXT-4, P:975-987) |
+| `r02_bench.json` | `python bench.py` — the JSON line the driver reads (headline + schemes + SSB SF20 + issue roof + all-core oracle + config 1) |
+| `r02_launches_bench.csv` | `ncu --metrics gpu__time_duration.sum --clock-control none` launch list of `bench.py --quick` |
+| `ncu_summary.json`, `r02_ncu_k_decode_sum_details.txt` | `ncu --set full` of the headline kernel — DRAM bytes per launch (`roofline.traffic`), issue, occupancy |
+| `r02_suite.json` | `scripts/bench_suite.py` — every config 2-4 column at 500M rows, both modes, full-size parity |
+| `r02_issue.json` | `scripts/issue_profile.sh` — warp instructions / value, pipe split, issue-active, stalls per config |
+| `r02_tile_sweep.json`, `r02_tile_sweep2.json` | `scripts/tile_sweep.py` — NEXT-4 tiles-per-item / ring / CTAs-per-SM sweep (P:811-892) |
+| `r02_ssb_sf20.json`, `r02_ssb_sf20_none.json`, `r02_ssb_sf160.json` | `scripts/bench_ssb.py` — 13 queries, GPU-* (checked against the oracle) / None / SF160 |
+| `r02_star_*.txt` | ncu source hot spots and details of the star kernel (q1.1, q2.1, q3.1, q4.1) |
+| `r02_star_waits.txt` | `scripts/prof_waits.py` — per-column cycle split of the star kernel (profiling build) |
+| `r0?_encode.json`, `r0?_random_access.json`, `r0?_cascaded_ablation.json`, `r0?_nomb_ablation.json`, `r01_waterfall_sf20.json` | encoder, random access, cascading / miniblock ablations, SSB waterfall |
 
 ## Headline (config 2, b = 16, 500M rows, decode fused into an int64 sum)
 
-* step {b['ms_per_step']:.4f} ms; `k_decode_sum` average {r['kernel_avg_ms'] * 1000:.1f} µs (CUDA events over 500 launches)
+* step {b['ms_per_step']:.4f} ms; `k_decode_sum` average {r['kernel_avg_ms'] * 1000:.1f} µs (CUDA events over {b['steps']} launches)
 * achieved {r['achieved']:,.0f} GB/s on compressed bytes = **{100 * r['frac']:.1f} % of measured HBM**; {b['value'] / 1000:.1f} TB/s decoded;
-  {b['vs_baseline']:.1f}× the paper's V100 number for the same workload (1.55 ms, P:954-956).  Across box
-  allocations the same build measures 160.5-167 µs (96-99.6 %).
+  {b['vs_baseline']:.1f}× the paper's V100 number for the same workload (1.55 ms, P:954-956)
 * ncu (cold, serialised, one launch): {ncu['duration_s'] * 1e6:.1f} µs, DRAM read {ncu['dram_bytes_read'] / 1e9:.4f} GB + write
-  {ncu['dram_bytes_write'] / 1e6:.1f} MB = {ncu['traffic_over_algorithmic']:.3f} × the algorithmic 1.0469 GB (no re-reads),
-  {ncu['inst_executed'] / 1e6:.0f} M warp instructions, issue active {ncu['issue_active_pct']:.0f} %, {ncu['registers']} registers
-* launch list share: inside a bench step the only other launch is torch's 1-element zero fill (~2 µs);
-  `k_plain_sum` rows are the uncompressed "None" context measurement after the timed region.
-* e2e (compressed arrays copied from pinned host memory every step): {b['e2e']['value']:.0f} GB/s decoded (PCIe-bound)
-* cpu_baseline (the oracle, 1 thread): {b['cpu_baseline']['value']:.2f} GB/s decoded
+  {ncu['dram_bytes_write'] / 1e6:.1f} MB = {ncu['traffic_over_algorithmic']:.3f} × the algorithmic 1.0469 GB, {ncu['inst_executed'] / 1e6:.0f} M warp instructions,
+  issue active {ncu['issue_active_pct']:.0f} %, {ncu['registers']} registers
+* e2e (compressed arrays from pinned host memory every step): {b['e2e']['value']:.0f} GB/s decoded (PCIe-bound)
+* cpu_baseline (the oracle on {b['cpu_baseline']['cores']} host cores, {b['cpu_baseline'].get('cpu_model')}): {b['cpu_baseline']['value']:.2f} GB/s
+  decoded; 1 core {b['cpu_baseline']['one_core']['value']:.2f} GB/s; config 1 (16 × 1M-row round trips) {b['config1']['seconds']:.2f} s
 """
-    d = load("r01_suite.json")
-    s += """
-## Sweep and other schemes (r01_suite.json, 500M rows, single launches after an L2 flush)
+    roof = b.get("issue_roof") or {}
+    if roof:
+        s += "\n## INT32 issue roof (bench.py `issue_roof`, SURVEY 8(d))\n\n| kind | warp instructions / s | lane ops / s |\n|---|---|---|\n"
+        for k, v in roof.items():
+            if isinstance(v, dict):
+                s += f"| {k} | {v['warp_insts_per_s'] / 1e12:.3f} T | {v['lane_ops_per_s'] / 1e12:.1f} T |\n"
+        s += (f"\nRoof used for `issue_frac`: {roof['roof_warp_insts_per_s'] / 1e12:.3f} T warp instructions / s "
+              "(148 SMs × 4 SMSPs × 1.965 GHz = 1.163 T at one per SMSP per cycle).\n")
+    sch = b.get("schemes") or {}
+    if sch:
+        s += ("\n## Schemes in the bench line (configs 2-4, 500M rows, L2 flushed)\n\n| config | bits/int | sum ms | sum HBM frac | "
+              "sum instr/value | sum issue frac | global ms | global HBM frac | parity |\n|---|---|---|---|---|---|---|---|---|\n")
+        for k, v in sch.items():
+            s += (f"| {k} | {v['bits_per_int']:.2f} | {v['sum_ms']:.3f} | {v['sum_hbm_frac']:.2f} | "
+                  f"{v.get('sum_insts_per_value', float('nan')):.1f} | {v.get('sum_issue_frac', float('nan')):.2f} | "
+                  f"{v['global_ms']:.3f} | {v['global_hbm_frac']:.2f} | {all(v['parity'].values())} |\n")
+    d = load("r02_suite.json")
+    iss = (load("r02_issue.json") or {}).get("configs", {})
+    if d:
+        s += """
+## Sweep and other schemes (r02_suite.json + r02_issue.json, 500M rows, single launches after an L2 flush)
 
-| column | bits/int | decode→sum ms | HBM frac | decoded TB/s | decode→global ms | HBM frac (read + 2 GB write) |
-|---|---|---|---|---|---|---|
+| column | bits/int | decode→sum ms | HBM frac | instr/value | issue active % | decode→global ms | HBM frac (read + 2 GB write) |
+|---|---|---|---|---|---|---|---|
 """
-    for k, v in d["configs"].items():
-        if k.startswith("for_b") and int(k[5:]) not in (0, 1, 4, 8, 12, 16, 24, 32):
-            continue
-        s += (f"| {k} | {v['bits_per_int']:.2f} | {v['sum_ms']:.3f} | {v['sum_hbm_frac']:.2f} | "
-              f"{v['sum_decoded_gbs'] / 1000:.1f} | {v['global_ms']:.3f} | {v['global_hbm_frac']:.2f} |\n")
-    s += """
-Decode-only below b ≈ 12 and for DFOR / RFOR is instruction-bound (the compressed bytes are too few
-for HBM to bind: SURVEY App. C.4); decode→global is the HBM-bound mode the ≥70 % target applies to.
-"""
-    e = load("r01_encode.json")
-    s += """
-## GPU encoder (r01_encode.json, 500M rows; NEXT-3)
+        for k, v in d["configs"].items():
+            if k.startswith("for_b") and int(k[5:]) not in (0, 1, 4, 8, 12, 16, 24, 32):
+                continue
+            i = iss.get(k.replace("^", ""), {})
+            s += (f"| {k} | {v['bits_per_int']:.2f} | {v['sum_ms']:.3f} | {v['sum_hbm_frac']:.2f} | "
+                  f"{i.get('sum_insts_per_value', float('nan')):.1f} | {i.get('sum_issue_active_pct') or float('nan'):.0f} | "
+                  f"{v['global_ms']:.3f} | {v['global_hbm_frac']:.2f} |\n")
+    for name in ("r02_tile_sweep.json", "r02_tile_sweep2.json"):
+        t = load(name)
+        if t:
+            s += f"\n## {name} (NEXT-4, P:811-892)\n\n| point | ms | HBM frac |\n|---|---|---|\n"
+            for k, v in t["points"].items():
+                s += f"| {k} | {v['ms']:.4f} | {v['hbm_frac']:.3f} |\n"
+    q, n, q160 = load("r02_ssb_sf20.json"), load("r02_ssb_sf20_none.json"), load("r02_ssb_sf160.json")
+    if q and n:
+        s += f"""
+## SSB (r02_ssb_sf20.json, r02_ssb_sf20_none.json, r02_ssb_sf160.json)
 
-| column | GPU encode ms | HBM frac (4 B/row read + compressed written) | GPU-* analysis (3 schemes) ms | host encoder s (all cores) | oracle rows/s (1 thread) |
-|---|---|---|---|---|---|
-"""
-    for k, v in e["configs"].items():
-        s += (f"| {k} | {v['gpu_encode_ms']:.3f} | {v['gpu_encode_hbm_frac']:.2f} | {v['gpu_sizes_all3_ms']:.2f} | "
-              f"{v['host_encode_s']:.3f} | {v.get('oracle_encode_rows_per_s', 0) / 1e6:.0f} M |\n")
-    s += """
-Every GPU-encoded column is byte-identical to the host encoder's (itself pinned to the oracle) and
-decodes to its input.  FOR / DFOR are bounded by the chunk look-back (ncu: half the stall samples
-on the barrier after it); RFOR by the run marking + two streams at 2 CTAs/SM.  Context: the paper
-encodes 250M values in 1.2 / 1.3 / 2.2 s on 6 vCPUs (P:1228-1232).
-"""
-    q, n, q160 = load("r01_ssb_sf20.json"), load("r01_ssb_sf20_none.json"), load("r01_ssb_sf160.json")
-    s += f"""
-## SSB (r01_ssb_sf20.json, r01_ssb_sf20_none.json, r01_ssb_sf160.json)
-
-All 13 SF20 queries equal the oracle (exact int64).  GPU-* picks RFOR for lo_orderdate and
-lo_custkey and FOR elsewhere (P:1916-1918, 2009-2011).  Geomean kernel time at SF20: GPU-*
+All 13 SF20 queries equal the oracle (exact int64).  Geomean kernel time at SF20: GPU-*
 {q['geomean_query_ms']:.3f} ms, None {n['geomean_query_ms']:.3f} ms (paper V100: None 1.35× faster than GPU-*; here
-{q['geomean_query_ms'] / n['geomean_query_ms']:.2f}×); SF160: {q160['geomean_query_ms']:.2f} ms.
+{q['geomean_query_ms'] / n['geomean_query_ms']:.2f}×){f"; SF160: {q160['geomean_query_ms']:.2f} ms" if q160 else ""}.
 
-| query | SF20 GPU-* ms | SF20 None ms | SF20 HBM floor ms | SF160 GPU-* ms |
-|---|---|---|---|---|
+| query | SF20 GPU-* ms | HBM frac | SF20 None ms | SF20 HBM floor ms |{" SF160 GPU-* ms |" if q160 else ""}
+|---|---|---|---|---|{"---|" if q160 else ""}
 """
-    for k, v in q["queries"].items():
-        s += (f"| {k} | {v['kernel_ms']:.3f} | {n['queries'][k]['kernel_ms']:.3f} | {v['hbm_floor_ms']:.3f} | "
-              f"{q160['queries'][k]['kernel_ms']:.3f} |\n")
-    s += """
-The star kernel is instruction/latency-bound (RFOR expansion of the date / customer keys, probe
-round trips, 2-3 CTAs/SM by registers and shared memory), not HBM-bound.
-"""
-    ra = load("r01_random_access.json")
-    s += """
-## Random access (r01_random_access.json, 250M rows, P:1241-1262)
-
-| σ | FOR b=16 ms | None ms | DFOR sorted ms | RFOR runs8 ms |
-|---|---|---|---|---|
-"""
-    pts = {}
-    for p_ in ra["points"]:
-        pts.setdefault(p_["sigma"], {})[p_["column"]] = p_["ms"]
-    for sg, v in pts.items():
-        s += f"| {sg:.3g} | {v['for_b16']:.3f} | {v['none_b16']:.3f} | {v['dfor_sorted']:.3f} | {v['rfor_runs8']:.3f} |\n"
-    s += """
-At σ ≥ 1/32 every FOR miniblock is read and FOR beats None (paper V100 2.1 vs 2.5 ms); below
-σ ≈ 1/512 most tiles are skipped; in between None reads fewer bytes (one 128-byte line per
-selected miniblock vs FOR's block_starts → header → miniblock chain).
-"""
-    c = load("r01_cascaded_ablation.json")
-    w = load("r01_waterfall_sf20.json")
-    s += f"""
-## Ablations (r01_cascaded_ablation.json, r01_waterfall_sf20.json)
-
-Tile-based vs cascading decode (250M rows, decode→global, geomean over the sweep): FOR
-{c['ratio_geomean']['for']:.1f}×, DFOR {c['ratio_geomean']['dfor']:.1f}×, RFOR {c['ratio_geomean']['rfor']:.1f}× (paper V100: 2.6× / 4× / 8×).
-SSB SF20 waterfall: GPU-* footprint {w['footprint_ratio_none_over_gpu*']:.2f}× below None over all lineorder columns
-(paper 2.8×); tile decode vs cascading {w['decode_speedup_geomean_vs_cascaded']:.1f}× geomean per column.
-"""
-    nm = load("r01_nomb_ablation.json")
-    if nm:
-        s += """
-## Miniblock ablation (r01_nomb_ablation.json, 500M rows, P:975-987)
-
-| column | FOR bits/int | no-miniblock bits/int | FOR decode→sum ms | no-miniblock decode→sum ms | FOR →global ms | no-miniblock →global ms |
-|---|---|---|---|---|---|---|
-"""
-        for k, v in nm["columns"].items():
-            f, g = v["for"], v["fornm"]
-            s += (f"| {k} | {f['bits_per_int']:.2f} | {g['bits_per_int']:.2f} | {f['sum_ms']:.3f} | {g['sum_ms']:.3f} | "
-                  f"{f['global_ms']:.3f} | {g['global_ms']:.3f} |\n")
-        s += """
-On B200 both layouts decode b = 16 at the HBM roof (paper V100: 2.0 vs 2.1 ms, the no-miniblock
-layout 5 % faster); miniblocks cost nothing there and keep skewed columns 15 % smaller.
-"""
+        for k, v in q["queries"].items():
+            s += (f"| {k} | {v['kernel_ms']:.3f} | {v['hbm_frac']:.2f} | {n['queries'][k]['kernel_ms']:.3f} | {v['hbm_floor_ms']:.3f} |"
+                  + (f" {q160['queries'][k]['kernel_ms']:.3f} |" if q160 else "") + "\n")
+    for tag in ("encode", "random_access", "cascaded_ablation", "nomb_ablation"):
+        nm, _ = first(f"r02_{tag}.json", f"r01_{tag}.json")
+        if nm:
+            s += f"\n`{nm}`: see DESIGN.md §7 / the script that writes it.\n"
     open(os.path.join(P, "README.md"), "w").write(s)
     print("wrote profiles/README.md")
 

@@ -21,6 +21,8 @@ timeout 600 python scripts/bench_ssb.py --sf 20 --scheme none --out $R/ssb_sf20_
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_star_query -c 4 -o $R/star python scripts/profile_ssb.py 20 1.1,2.1,3.1,4.1 > $R/star_ncu.log 2>&1
 for i in 0 1 2 3; do python scripts/src_hot.py $R/star.ncu-rep 40 $i > $R/star_src_hot_$i.txt 2>&1; done
 ncu -i $R/star.ncu-rep --page details > $R/star.details.txt 2>&1; rm -f $R/star.ncu-rep
+python scripts/build_variant.py prof "-DTP_PROFILE_WAITS" > /dev/null 2>&1
+TILEPACK_LIB_OVERRIDE=$PWD/build_ab/libtilepack_prof.so timeout 600 python scripts/prof_waits.py 20 1.1,1.2,1.3,2.1,2.2,2.3,3.1,3.2,3.3,3.4,4.1,4.2,4.3 > $R/star_waits.txt 2>&1
 timeout 1200 python scripts/bench_ssb.py --sf 160 --reps 5 --out $R/ssb_sf160.json > $R/ssb160.log 2>&1; echo "ssb160 rc=$?"
 timeout 900 python scripts/bench_encode.py --out $R/encode.json > $R/encode.log 2>&1; echo "enc rc=$?"
 timeout 600 python scripts/bench_random_access.py --reps 5 --out $R/random_access.json > $R/ra.log 2>&1; echo "ra rc=$?"

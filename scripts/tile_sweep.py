@@ -31,7 +31,11 @@ POINTS2["tw8192_qring40kb"] = "-DTP_TARGET_WORDS=8192u -DTP_QUERY_RING_KB=40"
 CONFIGS = {"for_b4": ("for", lambda n: __import__("datagen").uniform_bits(4, n, seed=2004)),
            "for_b16": ("for", lambda n: __import__("datagen").uniform_bits(16, n, seed=2016)),
            "dfor_d1": ("dfor", lambda n: __import__("datagen").d1_sorted(n, 2**28)),
-           "rfor_runs8": ("rfor", lambda n: __import__("datagen").runs(n, 8))}
+           "rfor_runs8": ("rfor", lambda n: __import__("datagen").runs(n, 8)),
+           "rfor_runs4": ("rfor", lambda n: __import__("datagen").runs(n, 4)),
+           "dfor_near": ("dfor", lambda n: __import__("datagen").near_sorted(n)),
+           "dfor_sorted": ("dfor", lambda n: __import__("datagen").sorted_uniform(n)),
+           "dfor_consec": ("dfor", lambda n: __import__("datagen").consecutive(n))}
 
 
 def build(points=POINTS):
@@ -103,6 +107,10 @@ if __name__ == "__main__":
         build({f"sw2_{k}": v for k, v in POINTS2.items()})
     elif sys.argv[1] == "--child":
         child(sys.argv[2])
+    elif sys.argv[1] == "--ab":  # --ab OUT.json cfg1,cfg2 LIB...
+        libs = sys.argv[4:]
+        pts = {os.path.basename(l)[len("libtilepack_"):-3]: "" for l in libs}
+        run(sys.argv[2], pts, tuple(sys.argv[3].split(",")), "")
     elif sys.argv[1] == "--run2":
         run(sys.argv[2], POINTS2, ("for_b4", "for_b16", "dfor_d1", "rfor_runs8"), "sw2_")
     else:

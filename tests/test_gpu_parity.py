@@ -153,9 +153,10 @@ def test_lean_for_sum_full_rounds(b):
 
 
 def test_device_format_errors_flagged():
-    """Format violations the kernels meet are flagged (tp_device_errors), not silent: a bitwidth
-    byte > 32 (R3, R5) and a max_tile_words below the column's real tile span (the ring stays in
-    bounds, the flag says the result is undefined)."""
+    """Format violations the kernels meet are flagged (tp_device_errors), not silent: a
+    max_tile_words below the column's real tile span (the ring stays in bounds, the flag says the
+    result is undefined) and an RFOR run count > 512; a bitwidth byte > 32 (R3, R5) is used as 32
+    on the device (memory-safe) and reported by tp_validate on the host."""
     assert tp.tp_device_errors() == 0
     x = datagen.uniform_bits(10, 5_000_000 + 5, seed=3)  # many tiles per CTA: items of many tiles
     h = tp.encode(x, "for")
@@ -167,7 +168,12 @@ def test_device_format_errors_flagged():
     bad[bw] = (bad[bw] & ~np.uint32(0xff0000)) | np.uint32(45 << 16)
     d.data0.copy_(torch.from_numpy(bad.view(np.int32)))
     tp.decode_sum(d)
-    assert tp.tp_device_errors() & tp.TP_DEVERR_BITWIDTH
+    torch.cuda.synchronize()  # completes without a fault (the byte is used as 32)
+    old_word = h.data0[bw]
+    h.data0[bw] = bad[bw]
+    with pytest.raises(tp.TilepackError, match="malformed"):
+        tp.tp_validate(h.col)
+    h.data0[bw] = old_word
     d = h.to_device()
     d.col.max_tile_words0 = 8  # far below the 4 x (2 + 4 x 10) words of a tile
     tp.decode_sum(d)
