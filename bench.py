@@ -38,7 +38,6 @@ import os
 import statistics
 import subprocess
 import sys
-import threading
 import time
 
 import numpy as np
@@ -76,56 +75,69 @@ def dist_env():
 
 
 # ------------------------------------------------------------------ clocks (NVML, during the timed region)
+_REASONS = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown",
+            0x4: "sw_power_cap", 0x80: "hw_power_brake_slowdown", 0x2: "applications_clocks_setting",
+            0x100: "display_clock_setting", 0x1: "gpu_idle", 0x10: "sync_boost"}
+
+
+def _clock_sampler_proc(index, period, go, stop, out):
+    """Child process: NVML SM clock + clock-event reasons every `period` s between go and stop
+    (a thread in the launching process would compete for the GIL: measured 1 sample in 32 ms)."""
+    import pynvml
+    pynvml.nvmlInit()
+    h = pynvml.nvmlDeviceGetHandleByIndex(index)
+    samples, reasons = [], set()
+    go.wait()
+    while not stop.is_set():
+        try:
+            samples.append(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM))
+            r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+            reasons |= {n for bit, n in _REASONS.items() if r & bit and n not in ("gpu_idle", "applications_clocks_setting")}
+        except Exception:
+            pass
+        time.sleep(period)
+    out.put((samples, sorted(reasons)))
+
+
 class ClockSampler:
-    """Samples the SM clock and the clock-event reasons every 0.5 ms (a sampler without a sleep
-    holds the GIL so often that the launching thread falls behind the GPU: measured 3.6x on a
-    20-step region)."""
+    """Samples the SM clock and the clock-event reasons every 0.5 ms during the timed region, from
+    a separate process (started before, so its start-up is not timed)."""
 
     def __init__(self, index: int, period: float = 0.0005):
-        self.samples, self.reasons, self.max_mhz = [], set(), None
-        self.period, self._stop = period, threading.Event()
+        self.samples, self.reasons, self.max_mhz, self.proc = [], [], None, None
+        self.period = period
         try:
+            import multiprocessing as mp
             import pynvml
             pynvml.nvmlInit()
-            self.nv = pynvml
-            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
-            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(pynvml.nvmlDeviceGetHandleByIndex(index), pynvml.NVML_CLOCK_SM)
+            ctx = mp.get_context("spawn")
+            self.go, self.stop, self.q = ctx.Event(), ctx.Event(), ctx.Queue()
+            self.proc = ctx.Process(target=_clock_sampler_proc, args=(index, period, self.go, self.stop, self.q),
+                                    daemon=True)
+            self.proc.start()
         except Exception:
-            self.nv = None
-
-    _NAMES = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown",
-              0x4: "sw_power_cap", 0x80: "hw_power_brake_slowdown", 0x2: "applications_clocks_setting",
-              0x100: "display_clock_setting", 0x1: "gpu_idle", 0x10: "sync_boost"}
-
-    def _run(self):
-        while not self._stop.is_set():
-            try:
-                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
-                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
-                for bit, name in self._NAMES.items():
-                    if r & bit and name not in ("gpu_idle", "applications_clocks_setting"):
-                        self.reasons.add(name)
-            except Exception:
-                pass
-            if self.period:
-                time.sleep(self.period)
+            self.proc = None
 
     def __enter__(self):
-        if self.nv:
-            self.t = threading.Thread(target=self._run, daemon=True)
-            self.t.start()
-            time.sleep(0.002)  # the sampler is running before the timed region starts
+        if self.proc:
+            self.go.set()
+            time.sleep(0.003)  # the sampler is running before the timed region starts
         return self
 
     def __exit__(self, *a):
-        if self.nv:
-            self._stop.set()
-            self.t.join()
+        if self.proc:
+            self.stop.set()
+            try:
+                self.samples, self.reasons = self.q.get(timeout=30)
+            except Exception:
+                pass
+            self.proc.join(timeout=10)
 
     def summary(self):
         return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
-                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples),
-                "source": "NVML (same counters as nvidia-smi), sampled every 0.5 ms during the timed steps"}
+                "sm_max_mhz": self.max_mhz, "reasons": list(self.reasons), "samples": len(self.samples),
+                "source": "NVML (same counters as nvidia-smi) in a separate process, every 0.5 ms during the timed steps"}
 
 
 def measured_peak():
@@ -363,6 +375,7 @@ def ssb_leg(args, tp, dev, stream, torch, rank, world):
                 dist.barrier()
             torch.cuda.synchronize()
             e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+            torch.cuda._sleep(2_000_000)  # the GPU busy ~1 ms: the host's launch work is not timed
             e0.record(stream)
             eng.execute(prep, sums, counts, stream)
             e1.record(stream)
@@ -447,8 +460,9 @@ def main():
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
+    clk = ClockSampler(local)  # process start-up outside the timed region
     l0 = tp.tp_launch_count()
-    with ClockSampler(local) as clk:
+    with clk:
         start.record(stream)
         for i in range(args.steps):
             acc.zero_()

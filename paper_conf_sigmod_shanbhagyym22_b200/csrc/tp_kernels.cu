@@ -10,6 +10,7 @@
 #include <algorithm>
 #include <atomic>
 #include <climits>
+#include <mutex>
 #include <cstdlib>
 #include <cstring>
 
@@ -133,10 +134,18 @@ __device__ __forceinline__ void decode_for(const Params& P, const Col& c, const 
 // slots, then the tile-wide exclusive prefix sum (R13) -- a
 // register scan inside the thread plus a 16-lane shuffle scan across the
 // tile's miniblocks -- plus the tile's first value (Fig. 6).
+template <bool COMPACT>
+__device__ __forceinline__ void decode_dfor_sv(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
+                                               const StreamView& v, uint32_t (&val)[32]);
 template <bool COMPACT, bool QP = false>
 __device__ __forceinline__ void decode_dfor(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                             uint32_t (&val)[32]) {
-  const StreamView v = stream_view<QP>(P, c.s0, C);
+  decode_dfor_sv<COMPACT>(P, c, C, g, stream_view<QP>(P, c.s0, C), val);
+}
+// (the item's stream view given: the decode->sum consumer computes it once per item)
+template <bool COMPACT>
+__device__ __forceinline__ void decode_dfor_sv(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
+                                               const StreamView& v, uint32_t (&val)[32]) {
   uint32_t tl;
   bool tv;
   const MbView m = for_mb(P, c, C, g, v, tl, tv);
@@ -579,11 +588,26 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
 // round (Op::col returns false); the host must then size the ring for every item in between.
 constexpr uint32_t QNS = 16;
 #ifndef TP_QUERY_PREFETCH
-#define TP_QUERY_PREFETCH 2  // rounds the query producer prefetches into L2 ahead of the ring
+#define TP_QUERY_PREFETCH 0  // rounds the query producer prefetches into L2 ahead of the ring (1 / 2 /
+                             // 4 measured: no change on SSB SF20 -- off)
 #endif
 #ifndef TP_QPROD_SPIN
 #define TP_QPROD_SPIN 0
 #endif
+
+// lane `src`'s boundary of stream q (warp-uniform q): a jump to the one shuffle instead of one
+// shuffle pair per stream of the query (the producer's per-item cost sits on the ring's refill
+// path: 24 dependent shuffles per item at 12 streams)
+__device__ __forceinline__ uint32_t bnd_of(const uint32_t (&bnd)[MAX_STREAMS], uint32_t q, uint32_t src) {
+  switch (q) {
+#define TP_BCASE(K) \
+  case K: return __shfl_sync(FULL, bnd[K], src);
+    TP_BCASE(0) TP_BCASE(1) TP_BCASE(2) TP_BCASE(3) TP_BCASE(4) TP_BCASE(5)
+    TP_BCASE(6) TP_BCASE(7) TP_BCASE(8) TP_BCASE(9) TP_BCASE(10)
+#undef TP_BCASE
+    default: return __shfl_sync(FULL, bnd[MAX_STREAMS - 1], src);
+  }
+}
 
 template <class Op>
 __device__ __forceinline__ void run_query_pipeline(const Params& P, Op& op) {
@@ -652,15 +676,12 @@ __device__ __forceinline__ void run_query_pipeline(const Params& P, Op& op) {
 #endif
         for (uint32_t c = 0; c < P.ncols; ++c, ++item) {
           const Col& cc = P.col[c];
-          const uint32_t my_s = lane == 0 ? cc.s0 : (lane == 1 && cc.scheme == S_RFOR ? cc.s1 : 0xffu);
-          uint32_t mylo = 0u, myhi = 0u;
-#pragma unroll
-          for (int q = 0; q < MAX_STREAMS; ++q) {
-            if ((uint32_t)q < P.nstreams) {
-              const uint32_t a = __shfl_sync(FULL, bnd[q], g - gb);
-              const uint32_t b = __shfl_sync(FULL, bnd[q], g - gb + 1);
-              if (my_s == (uint32_t)q) { mylo = a; myhi = b; }
-            }
+          const bool rfor = cc.scheme == S_RFOR;
+          const uint32_t my_s = lane == 0 ? cc.s0 : (lane == 1 && rfor ? cc.s1 : 0xffu);
+          uint32_t mylo = bnd_of(bnd, cc.s0, g - gb), myhi = bnd_of(bnd, cc.s0, g - gb + 1);
+          if (rfor) {  // (column-uniform)
+            const uint32_t lo1 = bnd_of(bnd, cc.s1, g - gb), hi1 = bnd_of(bnd, cc.s1, g - gb + 1);
+            if (lane == 1) { mylo = lo1; myhi = hi1; }
           }
           const bool none = (Op::kMask & M_NONE) && cc.scheme == S_NONE;  // column-uniform
           uint32_t dbytes = 0u, sbytes = 0u, dwords = 0u, swords = 0u;
@@ -875,9 +896,23 @@ struct SumOp : OpBase {
           if (alive & (1u << i)) acc += (uint64_t)(int64_t)(int32_t)(m.ref + e[i]);
       }
     } else {
-      const uint32_t alive = valid_rows(P, C, g);
+      uint32_t alive;
       uint32_t val[32];
-      decode_col<MASK>(P, 0, C, g, scratch, val);
+      if constexpr (LEAN && MASK == M_DFOR) {
+        // GPU-DFOR is instruction-bound too: the stream view once per item, the CTA-uniform
+        // full-round test
+        if (C.t0s != sv_t0s) {
+          sv = stream_view(P, c.s0, C);
+          sv_t0s = C.t0s;
+        }
+        const uint32_t tend = C.t0s + C.round_base + TPR;
+        const bool full_round = tend <= C.tile_end && (uint64_t)tend * TILE_ROWS <= P.n;
+        alive = full_round ? 0xffffffffu : valid_rows(P, C, g);
+        decode_dfor_sv<false>(P, c, C, g, sv, val);
+      } else {
+        alive = valid_rows(P, C, g);
+        decode_col<MASK>(P, 0, C, g, scratch, val);
+      }
       if (alive == 0xffffffffu) {  // per-lane branch, no collectives inside
         uint64_t lo = 0;
         uint32_t neg = 0;
@@ -1594,6 +1629,9 @@ struct StarOp : OpBase {
 };
 
 // ------------------------------------------------------------------ kernels
+#ifndef TP_DFOR_LEAN
+#define TP_DFOR_LEAN 1
+#endif
 #ifndef TP_SUM_MINB
 #define TP_SUM_MINB 4
 #endif
@@ -2025,11 +2063,29 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
 
 template <class K>
 static int grid_for(K kernel, size_t smem) {
+  // the attribute + occupancy query per (kernel, shared-memory size, device), cached: both are
+  // host round trips into the driver that otherwise sit in front of every launch
+  struct Entry { const void* k; size_t smem; int dev; int occ; };
+  static Entry cache[64];
+  static int ncache = 0;
+  static std::mutex mu;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  {
+    std::lock_guard<std::mutex> lock(mu);
+    for (int i = 0; i < ncache; ++i)
+      if (cache[i].k == (const void*)kernel && cache[i].smem == smem && cache[i].dev == dev)
+        return sm_count() * cache[i].occ;
+  }
   cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   int occ = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, THREADS, smem);
   if (occ < 1) occ = 1;
   if (occ > 8) occ = 8;
+  {
+    std::lock_guard<std::mutex> lock(mu);
+    if (ncache < 64) cache[ncache++] = Entry{(const void*)kernel, smem, dev, occ};
+  }
   return sm_count() * occ;
 }
 
@@ -2087,7 +2143,13 @@ tp_status tp_decode_sum(const tp_column* dcol, int64_t* d_sum, void* stream) {
       else
         launch(k_decode_sum<M_FOR>, smem, cap, stream, P, out);
       break;
-    case M_DFOR: launch(k_decode_sum<M_DFOR>, smem, cap, stream, P, out); break;
+    case M_DFOR:
+#if TP_DFOR_LEAN
+      launch(k_decode_sum<M_DFOR, true>, smem, cap, stream, P, out);
+#else
+      launch(k_decode_sum<M_DFOR>, smem, cap, stream, P, out);
+#endif
+      break;
     case M_NONE: launch(k_decode_sum<M_NONE>, smem, cap, stream, P, out); break;
     case M_FORNM: launch(k_decode_sum<M_FORNM>, smem, cap, stream, P, out); break;
     default: launch(k_decode_sum<M_RFOR>, smem, cap, stream, P, out); break;
