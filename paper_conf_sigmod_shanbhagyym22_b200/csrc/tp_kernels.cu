@@ -2063,29 +2063,33 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
 
 template <class K>
 static int grid_for(K kernel, size_t smem) {
-  // the attribute + occupancy query per (kernel, shared-memory size, device), cached: both are
-  // host round trips into the driver that otherwise sit in front of every launch
-  struct Entry { const void* k; size_t smem; int dev; int occ; };
-  static Entry cache[64];
-  static int ncache = 0;
+  // the attribute + occupancy queries are host round trips into the driver in front of every
+  // launch: cached per (kernel, device) -- the largest dynamic shared-memory size set so far (a
+  // launch above it raises it) -- and per (kernel, size, device) for the occupancy
+  struct Attr { const void* k; int dev; size_t smem; };
+  struct Occ { const void* k; int dev; size_t smem; int occ; };
+  static Attr attrs[64];
+  static Occ occs[128];
+  static int nattr = 0, nocc = 0;
   static std::mutex mu;
   int dev = 0;
   cudaGetDevice(&dev);
-  {
-    std::lock_guard<std::mutex> lock(mu);
-    for (int i = 0; i < ncache; ++i)
-      if (cache[i].k == (const void*)kernel && cache[i].smem == smem && cache[i].dev == dev)
-        return sm_count() * cache[i].occ;
+  std::lock_guard<std::mutex> lock(mu);
+  int ai = -1;
+  for (int i = 0; i < nattr; ++i)
+    if (attrs[i].k == (const void*)kernel && attrs[i].dev == dev) ai = i;
+  if (ai < 0 || attrs[ai].smem < smem) {
+    cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (ai >= 0) attrs[ai].smem = smem;
+    else if (nattr < 64) attrs[nattr++] = Attr{(const void*)kernel, dev, smem};
   }
-  cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  for (int i = 0; i < nocc; ++i)
+    if (occs[i].k == (const void*)kernel && occs[i].dev == dev && occs[i].smem == smem) return sm_count() * occs[i].occ;
   int occ = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, THREADS, smem);
   if (occ < 1) occ = 1;
   if (occ > 8) occ = 8;
-  {
-    std::lock_guard<std::mutex> lock(mu);
-    if (ncache < 64) cache[ncache++] = Entry{(const void*)kernel, smem, dev, occ};
-  }
+  if (nocc < 128) occs[nocc++] = Occ{(const void*)kernel, dev, smem, occ};
   return sm_count() * occ;
 }
 
