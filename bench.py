@@ -80,15 +80,18 @@ _REASONS = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_s
             0x100: "display_clock_setting", 0x1: "gpu_idle", 0x10: "sync_boost"}
 
 
-def _clock_sampler_proc(index, period, go, stop, out):
+def _clock_sampler_proc(index, period, ready, go, stop, out):
     """Child process: NVML SM clock + clock-event reasons every `period` s between go and stop
     (a thread in the launching process would compete for the GIL: measured 1 sample in 32 ms)."""
     import pynvml
     pynvml.nvmlInit()
     h = pynvml.nvmlDeviceGetHandleByIndex(index)
     samples, reasons = [], set()
+    ready.set()
     go.wait()
-    while not stop.is_set():
+    first = True
+    while first or not stop.is_set():  # at least one sample, however short the region
+        first = False
         try:
             samples.append(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM))
             r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
@@ -112,10 +115,12 @@ class ClockSampler:
             pynvml.nvmlInit()
             self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(pynvml.nvmlDeviceGetHandleByIndex(index), pynvml.NVML_CLOCK_SM)
             ctx = mp.get_context("spawn")
-            self.go, self.stop, self.q = ctx.Event(), ctx.Event(), ctx.Queue()
-            self.proc = ctx.Process(target=_clock_sampler_proc, args=(index, period, self.go, self.stop, self.q),
-                                    daemon=True)
+            self.ready, self.go, self.stop, self.q = ctx.Event(), ctx.Event(), ctx.Event(), ctx.Queue()
+            self.proc = ctx.Process(target=_clock_sampler_proc,
+                                    args=(index, period, self.ready, self.go, self.stop, self.q), daemon=True)
             self.proc.start()
+            if not self.ready.wait(timeout=60):  # NVML up in the child before any timing starts
+                raise RuntimeError("clock sampler did not start")
         except Exception:
             self.proc = None
 

@@ -297,27 +297,15 @@ __device__ __forceinline__ void unpack_mb(const uint32_t* __restrict__ w, uint32
 // adds 32*ref once: sum(ref + e_i) = 32*ref + sum(e_i), exact in int64 because
 // every real value is ref + e_i without wrap, R4).  32-bit partial sums are
 // exact for B <= 27 (32 * (2^27 - 1) < 2^32).
-#ifndef TP_SUM_TREE
-#define TP_SUM_TREE 0
-#endif
 template <int B>
 __device__ __forceinline__ uint64_t sum_fixed(const uint32_t* __restrict__ w) {
   uint32_t e[32];
   unpack_fixed<B>(w, e);
   if constexpr (B <= 27) {
-#if TP_SUM_TREE
-    // four independent partial sums: the 32 adds form four short dependency chains instead of
-    // one (fixed-latency "wait" stalls were the top stall reason of the low-bitwidth sums)
-    uint32_t s[4] = {0u, 0u, 0u, 0u};
-#pragma unroll
-    for (int i = 0; i < 32; ++i) s[i & 3] += e[i];
-    return (s[0] + s[1]) + (s[2] + s[3]);
-#else
-    uint32_t s = 0;
+    uint32_t s = 0;  // (four independent partial sums measured no faster: the compiler's IADD3 tree)
 #pragma unroll
     for (int i = 0; i < 32; ++i) s += e[i];
     return s;
-#endif
   } else {
     uint64_t s = 0;
 #pragma unroll

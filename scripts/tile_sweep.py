@@ -50,8 +50,9 @@ def child(cfg):
     import numpy as np
     import torch
     from paper_conf_sigmod_shanbhagyym22_b200 import tilepack as tp
-    if cfg.isdigit():
-        scheme, gen = "for", (lambda n: __import__("datagen").uniform_bits(int(cfg), n, seed=2000 + int(cfg)))
+    if cfg.isdigit() or (cfg.startswith("for_b") and cfg not in CONFIGS):
+        b = int(cfg[5:] if cfg.startswith("for_b") else cfg)
+        scheme, gen = "for", (lambda n: __import__("datagen").uniform_bits(b, n, seed=2000 + b))
     else:
         scheme, gen = CONFIGS[cfg]
     x = gen(500_000_000)
