@@ -424,10 +424,15 @@ def main():
     import torch.distributed as dist
 
     rank, world, local = dist_env()
+    # TILEPACK_DIST_BACKEND=gloo: a functional check of the N > 1 path with several ranks on fewer
+    # GPUs (ranks share a device; NCCL needs one GPU per rank) -- never a measurement
+    backend = os.environ.get("TILEPACK_DIST_BACKEND", "nccl")
+    if backend != "nccl":
+        local %= max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        dist.init_process_group(backend, device_id=dev if backend == "nccl" else None)
     from paper_conf_sigmod_shanbhagyym22_b200 import tilepack as tp
 
     # ---------------- setup (untimed): generate + encode on the host, copy once

@@ -37,10 +37,15 @@ def main():
 
     rank, world = int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1))
     local = int(os.environ.get("LOCAL_RANK", 0))
+    # TILEPACK_DIST_BACKEND=gloo: a functional check of the N > 1 path with several ranks on fewer
+    # GPUs (ranks share a device; NCCL needs one GPU per rank) -- never a measurement
+    backend = os.environ.get("TILEPACK_DIST_BACKEND", "nccl")
+    if backend != "nccl":
+        local %= max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        dist.init_process_group(backend, device_id=dev if backend == "nccl" else None)
     t0 = time.time()
     db = gen.generate(args.sf, seed=5000, columns=gen.QUERY_COLUMNS)
     n = len(db["lineorder"]["lo_orderdate"])
