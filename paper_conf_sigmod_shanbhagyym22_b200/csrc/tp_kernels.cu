@@ -213,11 +213,50 @@ __device__ __forceinline__ uint32_t extract_at(const uint32_t* m, uint32_t p, ui
 __device__ __forceinline__ uint32_t rfor_a_pos(uint32_t s) { return s ^ ((s >> 3) & 0x1Cu); }
 __device__ __forceinline__ uint32_t rfor_f_pos(uint32_t s) { return s ^ (((s >> 7) & 1u) << 4); }
 
-// steps 1-3 for one block, C entries per lane
+#ifndef TP_RFOR_SPLIT
+#define TP_RFOR_SPLIT 2  // 128 < r <= 192: a 4-entry pass + a 1- / 2-entry tail pass instead of 8 entries
+                         // (2: also 64 < r <= 96 as 2 + 1 entries; runs of 8: -6 %, measured)
+#endif
+#ifndef TP_RFOR_WIN
+#define TP_RFOR_WIN 1  // a lane's C entries from one 64-bit window (runs of 4: -6 %, measured)
+#endif
+#ifndef TP_RFOR_BALLOT_CARRY
+#define TP_RFOR_BALLOT_CARRY 1  // carries by ballot + one shuffle (runs of 4: -2.5 %, SSB -0.3 %, measured)
+#endif
+#ifndef TP_GLOBAL_SPIN_INSTR
+#define TP_GLOBAL_SPIN_INSTR 0  // 1: decode->global of the instruction-bound DFOR / RFOR spins (0: parks, -0.6 %)
+#endif
+__device__ __forceinline__ void rfor_flag(uint8_t* F, uint32_t S) { F[rfor_f_pos(S)] = 1; }
+__device__ __forceinline__ void rfor_clear_flags(uint8_t* F, uint32_t lane) {
+  st_shared_v4(reinterpret_cast<uint32_t*>(F) + 4u * lane, 0u, 0u, 0u, 0u);
+}
+
+// the C consecutive b-bit fields [pos, pos + C) of miniblock words m (pos a multiple of C): one
+// 64-bit window of two words when they fit in it, else two words per field (extract_at)
 template <int C>
-__device__ __forceinline__ void rfor_scatter(const uint32_t* bV, const uint32_t* bL, uint32_t r, uint32_t lane,
-                                             uint32_t* A, uint8_t* F) {
-  const uint32_t e0 = C * lane, m = e0 >> 5, pos = e0 & 31u;
+__device__ __forceinline__ void extract_c(const uint32_t* m, uint32_t pos, uint32_t b, uint32_t mask,
+                                          uint32_t (&f)[C]) {
+  const uint32_t p0 = pos * b;
+#if TP_RFOR_WIN
+  if ((p0 & 31u) + C * b <= 64u) {
+    const uint32_t* w = m + (p0 >> 5);
+    const uint64_t win = (((uint64_t)w[1] << 32) | w[0]) >> (p0 & 31u);
+#pragma unroll
+    for (int k = 0; k < C; ++k) f[k] = (uint32_t)(win >> (k * b)) & mask;
+    return;
+  }
+#endif
+#pragma unroll
+  for (int k = 0; k < C; ++k) f[k] = extract_at(m, p0 + k * b, mask);
+}
+
+// steps 1-3 for entries [eb, eb + 32 C) of one block, C entries per lane (a lane's entries inside
+// one miniblock: C divides 32); rb = rows of the entries before eb.  Returns the pass's rows
+// (RET: only a pass followed by a tail pass needs them).
+template <int C, bool RET = false>
+__device__ __forceinline__ uint32_t rfor_scatter(const uint32_t* bV, const uint32_t* bL, uint32_t r, uint32_t lane,
+                                                 uint32_t* A, uint8_t* F, uint32_t eb = 0u, uint32_t rb = 0u) {
+  const uint32_t e0 = eb + C * lane, m = (e0 >> 5) & 15u, pos = e0 & 31u;
   const uint32_t refV = bV[1], refL = bL[1];  // references (FOR on both arrays)
   const uint4 wv = make_uint4(bV[2], bV[3], bV[4], bV[5]), wl = make_uint4(bL[2], bL[3], bL[4], bL[5]);
   const uint32_t bv = checked_bw(byte_of(wv, m)), bl = checked_bw(byte_of(wl, m));  // R2, R17
@@ -225,29 +264,53 @@ __device__ __forceinline__ void rfor_scatter(const uint32_t* bV, const uint32_t*
   const uint32_t* mV = bV + 6 + bytes_before(wv, m);
   const uint32_t* mL = bL + 6 + bytes_before(wl, m);
   const uint32_t mv = __funnelshift_lc(0xffffffffu, 0u, bv), ml = __funnelshift_lc(0xffffffffu, 0u, bl);
+  uint32_t fl[C], fv[C];
+  extract_c<C>(mL, pos, bl, ml, fl);  // Alg. 1 for the lane's C entries of each stream
   uint32_t len[C], incl[C];
   uint32_t run = 0u;
 #pragma unroll
   for (int k = 0; k < C; ++k) {  // 1. run lengths + lane-local inclusive scan
-    len[k] = e0 + k < r ? refL + extract_at(mL, (pos + k) * bl, ml) : 0u;
+    len[k] = e0 + k < r ? refL + fl[k] : 0u;
     run += len[k];
     incl[k] = run;
   }
-  const uint32_t base = warp_inclusive_scan(run, lane) - run;  // 2. rows before this lane's runs
+  extract_c<C>(mV, pos, bv, mv, fv);
+  const uint32_t wincl = warp_inclusive_scan(run, lane);
+  const uint32_t base = rb + wincl - run;  // 2. rows before this lane's runs
 #pragma unroll
   for (int k = 0; k < C; ++k) {  // 3. scatter values and start flags
     if (e0 + k < r) {
       const uint32_t S = (base + incl[k] - len[k]) & 511u;
-      A[rfor_a_pos(S)] = refV + extract_at(mV, (pos + k) * bv, mv);
-      F[rfor_f_pos(S)] = 1;
+      A[rfor_a_pos(S)] = refV + fv[k];
+      rfor_flag(F, S);
     }
   }
+  return RET ? __shfl_sync(FULL, wincl, 31) : 0u;
+}
+
+// steps 1-3 for one block of r runs: the fewest entries per lane that cover it (long runs: one)
+// SMALLC: also the C = 1 / 2 bodies (and tails) for blocks of few (long) runs
+template <bool SMALLC>
+__device__ __forceinline__ void rfor_block_scatter(const uint32_t* bV, const uint32_t* bL, uint32_t r, uint32_t lane,
+                                                   uint32_t* A, uint8_t* F) {
+  if (SMALLC && r <= 32u) rfor_scatter<1>(bV, bL, r, lane, A, F);
+  else if (SMALLC && r <= 64u) rfor_scatter<2>(bV, bL, r, lane, A, F);
+#if TP_RFOR_SPLIT >= 2
+  else if (SMALLC && r <= 96u) rfor_scatter<1>(bV, bL, r, lane, A, F, 64u, rfor_scatter<2, true>(bV, bL, r, lane, A, F));
+#endif
+  else if (r <= 128u) rfor_scatter<4>(bV, bL, r, lane, A, F);
+#if TP_RFOR_SPLIT
+  else if (SMALLC && r <= 160u) rfor_scatter<1>(bV, bL, r, lane, A, F, 128u, rfor_scatter<4, true>(bV, bL, r, lane, A, F));
+  else if (SMALLC && r <= 192u) rfor_scatter<2>(bV, bL, r, lane, A, F, 128u, rfor_scatter<4, true>(bV, bL, r, lane, A, F));
+#endif
+  else if (r <= 256u) rfor_scatter<8>(bV, bL, r, lane, A, F);
+  else rfor_scatter<16>(bV, bL, r, lane, A, F);
 }
 
 // steps 1-3 for both row blocks of the warp's round (block h -> scratch + h * RFOR_BLOCK_WORDS)
-// SMALLC: also the C = 1 / 2 bodies for blocks of few (long) runs -- single-column decodes
-// only: the query kernels keep the smaller code (their RFOR columns have short runs, and the
-// extra bodies cost the star kernels ~4 % through instruction-cache misses, measured)
+// SMALLC: single-column decodes only: the query kernels keep the smaller code (their RFOR columns
+// have short runs, and the extra bodies cost the star kernels ~4 % through instruction-cache
+// misses, measured)
 template <bool SMALLC = false, bool QP = false>
 __device__ __forceinline__ void rfor_scatter_round(const Params& P, const Col& c, const StageCtx& C, const Lane& g,
                                                    uint32_t* scratch) {
@@ -258,7 +321,7 @@ __device__ __forceinline__ void rfor_scatter_round(const Params& P, const Col& c
   for (uint32_t h = 0; h < 2; ++h) {
     uint32_t* A = scratch + h * RFOR_BLOCK_WORDS;
     uint8_t* F = reinterpret_cast<uint8_t*>(A + RFOR_A_WORDS);
-    st_shared_v4(reinterpret_cast<uint32_t*>(F) + 4u * lane, 0u, 0u, 0u, 0u);
+    rfor_clear_flags(F, lane);
     __syncwarp();
     const uint32_t tl = C.round_base + 2u * g.cw + h;
     if (C.t0s + tl >= C.tile_end) continue;  // warp-uniform; rows masked by the consumer
@@ -269,12 +332,7 @@ __device__ __forceinline__ void rfor_scatter_round(const Params& P, const Col& c
       tp_flag_error(4u);  // TP_DEVERR_RUNS
       r = 512u;
     }
-    // C = entries per lane: the fewest that cover the block's runs (long runs: one entry per lane)
-    if (SMALLC && r <= 32u) rfor_scatter<1>(bV, bL, r, lane, A, F);
-    else if (SMALLC && r <= 64u) rfor_scatter<2>(bV, bL, r, lane, A, F);
-    else if (r <= 128u) rfor_scatter<4>(bV, bL, r, lane, A, F);
-    else if (r <= 256u) rfor_scatter<8>(bV, bL, r, lane, A, F);
-    else rfor_scatter<16>(bV, bL, r, lane, A, F);
+    rfor_block_scatter<SMALLC>(bV, bL, r, lane, A, F);
   }
   __syncwarp();
 }
@@ -305,12 +363,20 @@ __device__ __forceinline__ RforChunk rfor_chunk(uint32_t* scratch, uint32_t lane
 __device__ __forceinline__ uint32_t rfor_carry(const RforChunk& k) {
   uint32_t has = k.mask != 0u;
   uint32_t last = has ? k.A[rfor_a_pos(32u * k.j + 31u - __clz(k.mask))] : 0u;
+#if TP_RFOR_BALLOT_CARRY
+  // the nearest earlier lane of the 16-lane block holding a run start (lane j = 0 always does:
+  // row 0 of a block starts a run) -- one ballot and one shuffle instead of a 4-step scan
+  const uint32_t lane = threadIdx.x & 31u;
+  const uint32_t hm = __ballot_sync(FULL, has) & ((1u << lane) - 1u) & (lane >= 16u ? 0xffff0000u : 0x0000ffffu);
+  return __shfl_sync(FULL, last, hm ? 31u - __clz(hm) : lane);
+#else
 #pragma unroll
   for (int d = 1; d < 16; d <<= 1) {
     const uint32_t yh = __shfl_up_sync(FULL, has, d, 16), yv = __shfl_up_sync(FULL, last, d, 16);
     if (k.j >= (uint32_t)d && !has) { has = yh; last = yv; }
   }
   return __shfl_up_sync(FULL, last, 1, 16);
+#endif
 }
 // step 4: forward fill of the chunk's 32 rows
 __device__ __forceinline__ void rfor_fill(const RforChunk& k, uint32_t carry, uint32_t (&val)[32]) {
@@ -941,7 +1007,9 @@ struct SumOp : OpBase {
 template <uint32_t MASK>
 struct GlobalOp : OpBase {
   static constexpr uint32_t kMask = MASK;
-  static constexpr bool kProducerSpin = true;  // HBM-bound (decoded rows are written back)
+  // HBM-bound (decoded rows are written back); the instruction-bound DFOR / RFOR expansions
+  // may park their waiting warps instead (TP_GLOBAL_SPIN_INSTR 0)
+  static constexpr bool kProducerSpin = TP_GLOBAL_SPIN_INSTR || (MASK != M_RFOR && MASK != M_DFOR);
   const CUtensorMap* tmap;
   int32_t* out;
   uint32_t full_rows32;  // n / 32: rows of the [n/32][32] tensor
@@ -963,9 +1031,10 @@ struct GlobalOp : OpBase {
     __syncwarp();
     const uint32_t l = g.lane;
 #pragma unroll
-    for (uint32_t q = 0; q < 8; ++q)
+    for (uint32_t q = 0; q < 8; ++q) {
       st_shared_v4(buf + l * 32u + ((q ^ (l & 7u)) << 2), val[4 * q], val[4 * q + 1], val[4 * q + 2],
                    val[4 * q + 3]);
+    }
     fence_proxy_async_smem();
     __syncwarp();
     const uint32_t mb0 = pair_tile * 16u;
@@ -1251,16 +1320,18 @@ struct StarOp : OpBase {
       const uint32_t mv = __funnelshift_lc(0xffffffffu, 0u, bv), ml = __funnelshift_lc(0xffffffffu, 0u, bl);
       uint32_t len[CC], val[CC];
       uint32_t run = 0u;
+      extract_c<CC>(mL, pos, bl, ml, len);
 #pragma unroll
       for (int k = 0; k < CC; ++k) {  // run lengths (scan step 1)
-        len[k] = e0 + k < r ? refL + extract_at(mL, (pos + k) * bl, ml) : 0u;
+        len[k] = e0 + k < r ? refL + len[k] : 0u;
         run += len[k];
       }
       const uint32_t incl = warp_inclusive_scan(run, lane);
       uint32_t S = 512u * h + rowbase + incl - run;  // round row of entry e0's run start
       rowbase += __shfl_sync(FULL, incl, 31);
+      extract_c<CC>(mV, pos, bv, mv, val);
 #pragma unroll
-      for (int k = 0; k < CC; ++k) val[k] = refV + extract_at(mV, (pos + k) * bv, mv);
+      for (int k = 0; k < CC; ++k) val[k] += refV;
       uint32_t pass = 0u;  // bit k: run k passes the column's role
       if (per_run) {
         if (range) {
@@ -1308,9 +1379,10 @@ struct StarOp : OpBase {
       const uint32_t* mL = bL + 6 + bytes_before(wl, m);
       const uint32_t ml = __funnelshift_lc(0xffffffffu, 0u, bl);
       uint32_t len[4], run = 0u;
+      extract_c<4>(mL, pos, bl, ml, len);
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
-        len[k] = e0 + k < r ? refL + extract_at(mL, (pos + k) * bl, ml) : 0u;
+        len[k] = e0 + k < r ? refL + len[k] : 0u;
         run += len[k];
       }
       const uint32_t incl = warp_inclusive_scan(run, lane);
@@ -1448,12 +1520,20 @@ struct StarOp : OpBase {
       rfor_runs<4>(bV, bL, r, h, c, range, per_run, need_ra, all_alive, RA, SB, PB, AW, lane);
     }
     __syncwarp();
-    const uint32_t sb = SB[lane], jj = lane & 15u;
+    const uint32_t sb = SB[lane];
     if (per_run) {
       // the passing bit of the run covering the row before this lane's first row: the status of
       // the last run start at or before it, a 16-lane segmented scan (row 0 of a block starts a run)
       const uint32_t pb = PB[lane];
       uint32_t has = sb != 0u, st = has ? (pb >> (31u - __clz(sb))) & 1u : 0u;
+#if TP_RFOR_BALLOT_CARRY
+      // the nearest earlier lane of the block with a run start (lane 0 of a block has one): its
+      // last start's passing bit, by two ballots
+      const uint32_t hm = __ballot_sync(FULL, has) & ((1u << lane) - 1u) & (lane >= 16u ? 0xffff0000u : 0xffffu);
+      const uint32_t stm = __ballot_sync(FULL, st);
+      const uint32_t cin = hm ? (stm >> (31u - __clz(hm))) & 1u : 0u;
+#else
+      const uint32_t jj = lane & 15u;
 #pragma unroll
       for (int d = 1; d < 16; d <<= 1) {
         const uint32_t yh = __shfl_up_sync(FULL, has, d, 16), ys = __shfl_up_sync(FULL, st, d, 16);
@@ -1461,6 +1541,7 @@ struct StarOp : OpBase {
       }
       const uint32_t up = __shfl_up_sync(FULL, st, 1, 16);
       const uint32_t cin = jj ? up : 0u;
+#endif
       // rows of passing runs: adding 1 right above each passing start (and above a virtual start
       // at row -1 carrying cin) into the continuation mask carries through the run's rows
       const uint64_t cont = (uint64_t)(~sb) << 1;
@@ -1778,7 +1859,7 @@ __global__ void __launch_bounds__(256) k_bitmap_sum(const __grid_constant__ Para
       for (uint32_t h = 0; h < 2; ++h) {
         uint32_t* A = scratch + h * RFOR_BLOCK_WORDS;
         uint8_t* F = reinterpret_cast<uint8_t*>(A + RFOR_A_WORDS);
-        st_shared_v4(reinterpret_cast<uint32_t*>(F) + 4u * lane, 0u, 0u, 0u, 0u);
+        rfor_clear_flags(F, lane);
         __syncwarp();
         const uint32_t th = 2u * pair + h;
         if (th >= P.ntiles || !((any >> (16u * h)) & 0xffffu)) continue;  // warp-uniform
@@ -1789,11 +1870,7 @@ __global__ void __launch_bounds__(256) k_bitmap_sum(const __grid_constant__ Para
           tp_flag_error(4u);  // TP_DEVERR_RUNS
           r = 512u;
         }
-        if (r <= 32u) rfor_scatter<1>(bV, bL, r, lane, A, F);
-        else if (r <= 64u) rfor_scatter<2>(bV, bL, r, lane, A, F);
-        else if (r <= 128u) rfor_scatter<4>(bV, bL, r, lane, A, F);
-        else if (r <= 256u) rfor_scatter<8>(bV, bL, r, lane, A, F);
-        else rfor_scatter<16>(bV, bL, r, lane, A, F);
+        rfor_block_scatter<true>(bV, bL, r, lane, A, F);
       }
       __syncwarp();
       const RforChunk k = rfor_chunk(scratch, lane);
