@@ -11,6 +11,7 @@
 #include <atomic>
 #include <climits>
 #include <mutex>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 
@@ -179,9 +180,14 @@ __device__ __forceinline__ void decode_dfor_sv(const Params& P, const Col& c, co
 //     nearest earlier thread (16-lane segmented scan), and forward-fills its rows.
 // A is stored XOR-swizzled by 16-byte quad so that the 16 threads' 128-bit reads of
 // their row chunks are conflict-free.  The result equals repeat(V, L) (R19).
+// per-warp scratch: the two blocks' A arrays side by side (4 KB: decode->global stages the warp's
+// 1024 decoded rows in the same bytes, so that a 4th CTA fits per SM), then their flag bytes
 constexpr uint32_t RFOR_A_WORDS = 512, RFOR_F_WORDS = 128;
-constexpr uint32_t RFOR_BLOCK_WORDS = RFOR_A_WORDS + RFOR_F_WORDS;
-constexpr uint32_t RFOR_SCRATCH_WORDS = 2 * RFOR_BLOCK_WORDS;
+constexpr uint32_t RFOR_SCRATCH_WORDS = 2 * (RFOR_A_WORDS + RFOR_F_WORDS);
+__device__ __forceinline__ uint32_t* rfor_A(uint32_t* scratch, uint32_t h) { return scratch + h * RFOR_A_WORDS; }
+__device__ __forceinline__ uint8_t* rfor_F(uint32_t* scratch, uint32_t h) {
+  return reinterpret_cast<uint8_t*>(scratch + 2 * RFOR_A_WORDS + h * RFOR_F_WORDS);
+}
 
 __device__ __forceinline__ uint32_t warp_inclusive_scan(uint32_t x, uint32_t lane) {
 #pragma unroll
@@ -307,7 +313,7 @@ __device__ __forceinline__ void rfor_block_scatter(const uint32_t* bV, const uin
   else rfor_scatter<16>(bV, bL, r, lane, A, F);
 }
 
-// steps 1-3 for both row blocks of the warp's round (block h -> scratch + h * RFOR_BLOCK_WORDS)
+// steps 1-3 for both row blocks of the warp's round (block h -> rfor_A / rfor_F(scratch, h))
 // SMALLC: single-column decodes only: the query kernels keep the smaller code (their RFOR columns
 // have short runs, and the extra bodies cost the star kernels ~4 % through instruction-cache
 // misses, measured)
@@ -319,8 +325,8 @@ __device__ __forceinline__ void rfor_scatter_round(const Params& P, const Col& c
   __syncwarp();  // a lagging lane may still read the previous column's expansion
 #pragma unroll 1
   for (uint32_t h = 0; h < 2; ++h) {
-    uint32_t* A = scratch + h * RFOR_BLOCK_WORDS;
-    uint8_t* F = reinterpret_cast<uint8_t*>(A + RFOR_A_WORDS);
+    uint32_t* A = rfor_A(scratch, h);
+    uint8_t* F = rfor_F(scratch, h);
     rfor_clear_flags(F, lane);
     __syncwarp();
     const uint32_t tl = C.round_base + 2u * g.cw + h;
@@ -346,8 +352,8 @@ struct RforChunk {
 __device__ __forceinline__ RforChunk rfor_chunk(uint32_t* scratch, uint32_t lane) {
   RforChunk k;
   k.j = lane & 15u;
-  k.A = scratch + (lane >> 4) * RFOR_BLOCK_WORDS;
-  const uint32_t* F = k.A + RFOR_A_WORDS;
+  k.A = rfor_A(scratch, lane >> 4);
+  const uint32_t* F = reinterpret_cast<const uint32_t*>(rfor_F(scratch, lane >> 4));
   const uint32_t fs = ((k.j >> 2) & 1u) << 2;  // flag quad swizzle (words)
   const uint4 f0 = *reinterpret_cast<const uint4*>(F + 8u * k.j + fs);
   const uint4 f1 = *reinterpret_cast<const uint4*>(F + 8u * k.j + (fs ^ 4u));
@@ -1015,20 +1021,28 @@ struct GlobalOp : OpBase {
   uint32_t full_rows32;  // n / 32: rows of the [n/32][32] tensor
   __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t,
                       uint32_t rc) {
+    // RFOR: the rows are staged in the expansion's own A arrays (1024-byte aligned: the host aligns
+    // the scratch), so the previous round's store must have read them before this round expands
+    constexpr bool OVERLAY = MASK == M_RFOR;
+    if (OVERLAY) {
+      if (g.lane == 0) bulk_wait_read<0>();
+      __syncwarp();
+    }
     uint32_t val[32];
     decode_col<MASK>(P, 0, C, g, scratch, val);
     const uint32_t pair_tile = C.t0s + C.round_base + 2u * g.cw;
     if (pair_tile >= C.tile_end) return;  // warp-uniform
-    uint32_t* buf = scratch + P.staging_off;
-    buf = reinterpret_cast<uint32_t*>((reinterpret_cast<uintptr_t>(buf) + 1023) & ~uintptr_t(1023));
-    // RFOR: one buffer (its shared-memory budget -- the expansion scratch -- is what keeps a 3rd
-    // CTA per SM; the expansion of the next round covers the store's read), else two
-    constexpr bool SINGLE = MASK == M_RFOR;
-    if (!SINGLE) buf += (rc & 1u) * 1024u;
-    if (g.lane == 0) {  // the store issued from this buffer earlier is done reading it
-      if (SINGLE) bulk_wait_read<0>(); else bulk_wait_read<1>();
+    uint32_t* buf;
+    if (OVERLAY) {
+      buf = scratch;
+      __syncwarp();  // every lane has read its chunk of A
+    } else {
+      buf = scratch + P.staging_off;
+      buf = reinterpret_cast<uint32_t*>((reinterpret_cast<uintptr_t>(buf) + 1023) & ~uintptr_t(1023));
+      buf += (rc & 1u) * 1024u;
+      if (g.lane == 0) bulk_wait_read<1>();  // the store issued from this buffer earlier is done reading it
+      __syncwarp();
     }
-    __syncwarp();
     const uint32_t l = g.lane;
 #pragma unroll
     for (uint32_t q = 0; q < 8; ++q) {
@@ -1857,8 +1871,8 @@ __global__ void __launch_bounds__(256) k_bitmap_sum(const __grid_constant__ Para
       __syncwarp();
 #pragma unroll 1
       for (uint32_t h = 0; h < 2; ++h) {
-        uint32_t* A = scratch + h * RFOR_BLOCK_WORDS;
-        uint8_t* F = reinterpret_cast<uint8_t*>(A + RFOR_A_WORDS);
+        uint32_t* A = rfor_A(scratch, h);
+        uint8_t* F = rfor_F(scratch, h);
         rfor_clear_flags(F, lane);
         __syncwarp();
         const uint32_t th = 2u * pair + h;
@@ -2130,7 +2144,7 @@ static tp_status build_params(const tp_column* cols, int ncols, uint32_t extra_s
   const uint32_t ring_kb = ncols > 1 ? TP_QUERY_RING_KB : (for_only ? TP_RING_KB : TP_QUERY_RING_KB);
   while (nstg > 2 && (size_t)nstg * P.stage_words * 4 > ring_kb * 1024) --nstg;
   P.nstages = nstg;
-  P.scratch_off = nstg * P.stage_words;
+  P.scratch_off = (nstg * P.stage_words + 255u) & ~255u;  // 1024-byte aligned (RFOR staging in scratch)
   P.agg_off = P.scratch_off + CONSUMER_WARPS * P.scratch_words_per_warp;
   P.bar_off = align4(P.agg_off + agg_words);
   if (P.bar_off & 1u) ++P.bar_off;  // 8-byte aligned barriers
@@ -2179,6 +2193,8 @@ static uint32_t scheme_mask(const Params& P) {
 template <class K, class... Args>
 static void launch(K kernel, size_t smem, int cap, void* stream, Args... args) {
   const int grid = std::max(1, std::min<int>(grid_for(kernel, smem), cap));
+  static const bool dbg = getenv("TILEPACK_DEBUG_LAUNCH") != nullptr;  // tuning: grid / smem per launch
+  if (dbg) fprintf(stderr, "TPLAUNCH grid=%d ctas_per_sm=%d smem=%zu\n", grid, grid / sm_count(), smem);
   kernel<<<grid, THREADS, smem, (cudaStream_t)stream>>>(args...);
 }
 
@@ -2249,8 +2265,8 @@ tp_status decode_global_impl(const tp_column* dcol, int32_t* d_out, bool raw, vo
   if (raw && dcol->scheme == TP_RFOR) return TP_EINVAL;
   Params P;
   size_t smem = 0;
-  // per warp: 2 x 4 KB swizzled staging (RFOR: 1) + 1 KB alignment slop
-  tp_status st = build_params(dcol, 1, (dcol->scheme == TP_RFOR ? 1024u : 2048u) + 256u, 0, P, smem);
+  // per warp: 2 x 4 KB swizzled staging + 1 KB alignment slop (RFOR: staged in its expansion scratch)
+  tp_status st = build_params(dcol, 1, dcol->scheme == TP_RFOR ? 0u : 2048u + 256u, 0, P, smem);
   if (st != TP_OK) return st;
   CUtensorMap tmap;
   memset(&tmap, 0, sizeof(tmap));

@@ -73,13 +73,15 @@ def main():
     for rep in range(reps):
         for lib in libs:
             name = os.path.basename(lib)
-            env = dict(os.environ, TILEPACK_LIB_OVERRIDE=os.path.abspath(lib))
+            env = dict(os.environ, TILEPACK_LIB_OVERRIDE=os.path.abspath(lib), TILEPACK_DEBUG_LAUNCH="1")
             o = subprocess.run([sys.executable, __file__, "--child", cfgs], env=env, capture_output=True, text=True)
             line = [x for x in o.stdout.splitlines() if x.startswith("RESULT")]
             if not line:
                 print(name, "FAILED", o.stderr[-800:], flush=True)
                 continue
             r = json.loads(line[0][7:])
+            launches = sorted({x for x in o.stderr.splitlines() if x.startswith("TPLAUNCH")})
+            print(name, "launch configs:", launches, flush=True)
             for cfg, v in r.items():
                 v["global_hbm_frac"] = (v["bytes"] + 2e9) / (v["global_ms"] / 1e3) / 1e9 / peak
                 allr.setdefault(name, {}).setdefault(cfg, []).append(v)
