@@ -192,6 +192,7 @@ struct alignas(64) Params {
   uint32_t agg_off;     // word offset of the per-CTA aggregation table
   uint32_t bar_off;     // word offset of the mbarriers (8-byte aligned)
   uint32_t ring_words;  // query pipeline: words of the byte ring (at smem offset 0)
+  uint32_t single_staging;  // decode->global: one staging buffer per warp (instruction-bound DFOR)
 };
 
 // ------------------------------------------------------------------ bit unpack

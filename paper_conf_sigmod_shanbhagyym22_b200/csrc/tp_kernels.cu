@@ -229,6 +229,12 @@ __device__ __forceinline__ uint32_t rfor_f_pos(uint32_t s) { return s ^ (((s >> 
 #ifndef TP_RFOR_BALLOT_CARRY
 #define TP_RFOR_BALLOT_CARRY 1  // carries by ballot + one shuffle (runs of 4: -2.5 %, SSB -0.3 %, measured)
 #endif
+#ifndef TP_GLOBAL_SINGLE_DFOR
+#define TP_GLOBAL_SINGLE_DFOR 1
+#endif
+#ifndef TP_DFOR_SINGLE_BITS
+#define TP_DFOR_SINGLE_BITS 3.0
+#endif
 #ifndef TP_GLOBAL_SPIN_INSTR
 #define TP_GLOBAL_SPIN_INSTR 0  // 1: decode->global of the instruction-bound DFOR / RFOR spins (0: parks, -0.6 %)
 #endif
@@ -1024,6 +1030,9 @@ struct GlobalOp : OpBase {
     // RFOR: the rows are staged in the expansion's own A arrays (1024-byte aligned: the host aligns
     // the scratch), so the previous round's store must have read them before this round expands
     constexpr bool OVERLAY = MASK == M_RFOR;
+    // GPU-DFOR of more than a few bits / int (instruction-bound): one staging buffer, so that a
+    // 4th CTA fits per SM (host's choice, warp-uniform)
+    const bool SINGLE = MASK == M_DFOR && P.single_staging;
     if (OVERLAY) {
       if (g.lane == 0) bulk_wait_read<0>();
       __syncwarp();
@@ -1039,8 +1048,12 @@ struct GlobalOp : OpBase {
     } else {
       buf = scratch + P.staging_off;
       buf = reinterpret_cast<uint32_t*>((reinterpret_cast<uintptr_t>(buf) + 1023) & ~uintptr_t(1023));
-      buf += (rc & 1u) * 1024u;
-      if (g.lane == 0) bulk_wait_read<1>();  // the store issued from this buffer earlier is done reading it
+      if (SINGLE) {
+        if (g.lane == 0) bulk_wait_read<0>();  // the previous store is done reading the buffer
+      } else {
+        buf += (rc & 1u) * 1024u;
+        if (g.lane == 0) bulk_wait_read<1>();  // the store issued from this buffer earlier is done reading it
+      }
       __syncwarp();
     }
     const uint32_t l = g.lane;
@@ -1182,6 +1195,24 @@ static inline uint32_t ht_slots(uint32_t ngroups) {
   uint32_t s = 256;
   while (s < HT_MAX_SLOTS && s < 2u * ngroups) s <<= 1;
   return s;
+}
+#ifndef TP_DENSE_PROBE_HINT
+#define TP_DENSE_PROBE_HINT 1
+#endif
+__device__ __forceinline__ int32_t probe_ld(const int32_t* p) { return __ldg(p); }
+// the dense probe of grouped queries (every alive row of a FOR / None column, the bulk of the
+// lookups of q2.x): L1::no_allocate + L2 evict_last (q2.x -9 %, q3.2 -2 %, measured; either hint
+// alone: no gain / +20 %; in the ungrouped kernel the changed code cost q1.1 4 %)
+__device__ __forceinline__ int32_t dense_probe_ld(const int32_t* p) {
+#if TP_DENSE_PROBE_HINT
+  int32_t v;
+  uint64_t pol;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+  return v;
+#else
+  return probe_ld(p);
+#endif
 }
 constexpr uint32_t STAR_RA_WORDS = 1024, STAR_SB_WORDS = 3 * 33 + 1;
 #ifndef TP_RFOR_CC8
@@ -1358,7 +1389,7 @@ struct StarOp : OpBase {
           for (int k = 0; k < CC; ++k) {
             const uint32_t key = val[k] - kmin;
             const bool live = e0 + k < r && key < tlen && (all_alive || run_alive(AW, Sk, len[k]));
-            val[k] = live ? (uint32_t)__ldg(T + key) : 0xffffffffu;  // payload, -1 = miss
+            val[k] = live ? (uint32_t)probe_ld(T + key) : 0xffffffffu;  // payload, -1 = miss
             Sk += len[k];
           }
 #pragma unroll
@@ -1469,7 +1500,7 @@ struct StarOp : OpBase {
         kill = (uint32_t)((int32_t)x - A->lo[c]) > (uint32_t)(A->hi[c] - A->lo[c]);
       } else if (role == TP_ROLE_PROBE) {
         const uint32_t kk = x - (uint32_t)A->key_min[c];
-        const int32_t p = kk < A->table_len[c] ? __ldg(A->table[c] + kk) : -1;
+        const int32_t p = kk < A->table_len[c] ? probe_ld(A->table[c] + kk) : -1;
         kill = p < 0;
         if (!kill && GROUPED && A->gmode[c]) {
           uint32_t* gp = G + 32u * i + j;
@@ -1615,7 +1646,7 @@ struct StarOp : OpBase {
 #pragma unroll
         for (int i = 0; i < 32; ++i) {
           const uint32_t kk = v[i] - kmin;
-          v[i] = ((m >> i) & 1u) && kk < len ? (uint32_t)__ldg(T + kk) : 0xffffffffu;
+          v[i] = ((m >> i) & 1u) && kk < len ? (uint32_t)(GROUPED ? dense_probe_ld(T + kk) : probe_ld(T + kk)) : 0xffffffffu;
         }
         dense_payload(c, v, G, lane);
       } else {
@@ -1690,7 +1721,7 @@ struct StarOp : OpBase {
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
           const uint32_t kk = xx[q] - kmin;
-          pl[q] = ok[q] && kk < len ? __ldg(T + kk) : -1;
+          pl[q] = ok[q] && kk < len ? probe_ld(T + kk) : -1;
         }
 #pragma unroll
         for (int q = 0; q < 4; ++q)
@@ -2265,9 +2296,16 @@ tp_status decode_global_impl(const tp_column* dcol, int32_t* d_out, bool raw, vo
   if (raw && dcol->scheme == TP_RFOR) return TP_EINVAL;
   Params P;
   size_t smem = 0;
-  // per warp: 2 x 4 KB swizzled staging + 1 KB alignment slop (RFOR: staged in its expansion scratch)
-  tp_status st = build_params(dcol, 1, dcol->scheme == TP_RFOR ? 0u : 2048u + 256u, 0, P, smem);
+  // per warp: 2 x 4 KB swizzled staging + 1 KB alignment slop (RFOR: staged in its expansion
+  // scratch).  GPU-DFOR at >= TP_DFOR_SINGLE_BITS bits / int takes one buffer -- 4 CTAs / SM
+  // instead of 3; measured on 500M rows: sorted-uniform (3.6 bits) -12 %, near-sorted (5.9) -6 %,
+  // but D1 (1.8, closer to the HBM roof) +5 %.  (A slop-free double buffer costs FOR b = 4 7 %.)
+  const bool single = TP_GLOBAL_SINGLE_DFOR && dcol->scheme == TP_DFOR && !raw &&
+                      (double)dcol->words0 * 32.0 >= TP_DFOR_SINGLE_BITS * (double)dcol->n;
+  const uint32_t staging = dcol->scheme == TP_RFOR ? 0u : (single ? 1024u : 2048u) + 256u;
+  tp_status st = build_params(dcol, 1, staging, 0, P, smem);
   if (st != TP_OK) return st;
+  P.single_staging = single ? 1u : 0u;
   CUtensorMap tmap;
   memset(&tmap, 0, sizeof(tmap));
   const uint32_t rows32 = (uint32_t)(dcol->n / 32);

@@ -80,7 +80,8 @@ def main():
                 print(name, "FAILED", o.stderr[-800:], flush=True)
                 continue
             r = json.loads(line[0][7:])
-            launches = sorted({x for x in o.stderr.splitlines() if x.startswith("TPLAUNCH")})
+            launches = [x[9:] for x in o.stderr.splitlines() if x.startswith("TPLAUNCH")]
+            launches = [x for i, x in enumerate(launches) if i == 0 or x != launches[i - 1]]  # per (cfg, mode)
             print(name, "launch configs:", launches, flush=True)
             for cfg, v in r.items():
                 v["global_hbm_frac"] = (v["bytes"] + 2e9) / (v["global_ms"] / 1e3) / 1e9 / peak
