@@ -319,6 +319,65 @@ __device__ __forceinline__ void rfor_block_scatter(const uint32_t* bV, const uin
   else rfor_scatter<16>(bV, bL, r, lane, A, F);
 }
 
+#ifndef TP_RFOR_PAIR
+#define TP_RFOR_PAIR 1  // single-column decodes: both blocks of a round in one pass (half-warp each)
+#endif
+// steps 1-3 for both blocks of the round at once: lanes 16 h .. 16 h + 15 take block h, entries
+// [eb, eb + 16 C) of it, C per lane (inside one miniblock); rb = rows of the block's entries before
+// eb.  One 16-lane segmented scan and one header decode per lane serve both blocks.  Returns the
+// rows of the half-warp's entries (RET).
+template <int C, bool RET = false>
+__device__ __forceinline__ uint32_t rfor_scatter_pair(const uint32_t* bV, const uint32_t* bL, uint32_t r,
+                                                      uint32_t lane, uint32_t* scratch, uint32_t eb = 0u,
+                                                      uint32_t rb = 0u) {
+  const uint32_t h = lane >> 4, e0 = eb + C * (lane & 15u), m = (e0 >> 5) & 15u, pos = e0 & 31u;
+  uint32_t* A = rfor_A(scratch, h);
+  uint8_t* F = rfor_F(scratch, h);
+  const uint32_t refV = bV[1], refL = bL[1];  // references (FOR on both arrays)
+  const uint4 wv = make_uint4(bV[2], bV[3], bV[4], bV[5]), wl = make_uint4(bL[2], bL[3], bL[4], bL[5]);
+  const uint32_t bv = checked_bw(byte_of(wv, m)), bl = checked_bw(byte_of(wl, m));  // R2, R17
+  const uint32_t* mV = bV + 6 + bytes_before(wv, m);  // miniblocks before m are full (R17)
+  const uint32_t* mL = bL + 6 + bytes_before(wl, m);
+  const uint32_t mv = __funnelshift_lc(0xffffffffu, 0u, bv), ml = __funnelshift_lc(0xffffffffu, 0u, bl);
+  uint32_t fl[C], fv[C];
+  extract_c<C>(mL, pos, bl, ml, fl);
+  uint32_t len[C], incl[C];
+  uint32_t run = 0u;
+#pragma unroll
+  for (int k = 0; k < C; ++k) {  // 1. run lengths + lane-local inclusive scan
+    len[k] = e0 + k < r ? refL + fl[k] : 0u;
+    run += len[k];
+    incl[k] = run;
+  }
+  extract_c<C>(mV, pos, bv, mv, fv);
+  const uint32_t wincl = seg16_inclusive_scan(run);
+  const uint32_t base = rb + wincl - run;  // 2. rows before this lane's runs (in its block)
+#pragma unroll
+  for (int k = 0; k < C; ++k) {  // 3. scatter values and start flags
+    if (e0 + k < r) {
+      const uint32_t S = (base + incl[k] - len[k]) & 511u;
+      A[rfor_a_pos(S)] = refV + fv[k];
+      rfor_flag(F, S);
+    }
+  }
+  return RET ? __shfl_sync(FULL, wincl, lane | 15u) : 0u;
+}
+// rm = the larger run count of the two blocks (warp-uniform): passes of 16 C entries per block
+__device__ __forceinline__ void rfor_pair_dispatch(const uint32_t* bV, const uint32_t* bL, uint32_t r, uint32_t rm,
+                                                   uint32_t lane, uint32_t* s) {
+  if (rm <= 16u) rfor_scatter_pair<1>(bV, bL, r, lane, s);
+  else if (rm <= 32u) rfor_scatter_pair<2>(bV, bL, r, lane, s);
+  else if (rm <= 64u) rfor_scatter_pair<4>(bV, bL, r, lane, s);
+  else if (rm <= 80u) rfor_scatter_pair<1>(bV, bL, r, lane, s, 64u, rfor_scatter_pair<4, true>(bV, bL, r, lane, s));
+  else if (rm <= 96u) rfor_scatter_pair<2>(bV, bL, r, lane, s, 64u, rfor_scatter_pair<4, true>(bV, bL, r, lane, s));
+  else if (rm <= 128u) rfor_scatter_pair<8>(bV, bL, r, lane, s);
+  else if (rm <= 144u) rfor_scatter_pair<1>(bV, bL, r, lane, s, 128u, rfor_scatter_pair<8, true>(bV, bL, r, lane, s));
+  else if (rm <= 160u) rfor_scatter_pair<2>(bV, bL, r, lane, s, 128u, rfor_scatter_pair<8, true>(bV, bL, r, lane, s));
+  else if (rm <= 192u) rfor_scatter_pair<4>(bV, bL, r, lane, s, 128u, rfor_scatter_pair<8, true>(bV, bL, r, lane, s));
+  else if (rm <= 256u) rfor_scatter_pair<16>(bV, bL, r, lane, s);
+  else rfor_scatter_pair<16>(bV, bL, r, lane, s, 256u, rfor_scatter_pair<16, true>(bV, bL, r, lane, s));
+}
+
 // steps 1-3 for both row blocks of the warp's round (block h -> rfor_A / rfor_F(scratch, h))
 // SMALLC: single-column decodes only: the query kernels keep the smaller code (their RFOR columns
 // have short runs, and the extra bodies cost the star kernels ~4 % through instruction-cache
@@ -329,6 +388,28 @@ __device__ __forceinline__ void rfor_scatter_round(const Params& P, const Col& c
   const StreamView vv = stream_view<QP>(P, c.s0, C, 0), vl = stream_view<QP>(P, c.s1, C, 1);
   const uint32_t lane = g.lane;
   __syncwarp();  // a lagging lane may still read the previous column's expansion
+  if (SMALLC && TP_RFOR_PAIR) {
+    // both blocks' flags cleared, then one pass over both (an invalid second block: no runs)
+    uint4* Fq = reinterpret_cast<uint4*>(rfor_F(scratch, 0));
+    Fq[lane] = make_uint4(0u, 0u, 0u, 0u);
+    Fq[lane + 32u] = make_uint4(0u, 0u, 0u, 0u);
+    __syncwarp();
+    const uint32_t tl0 = C.round_base + 2u * g.cw;
+    if (C.t0s + tl0 >= C.tile_end) return;  // warp-uniform; rows masked by the consumer
+    const bool v1 = C.t0s + tl0 + 1u < C.tile_end;
+    const uint32_t tl = tl0 + ((lane >> 4) && v1 ? 1u : 0u);
+    const uint32_t* bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
+    const uint32_t* bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
+    uint32_t r = bV[0];  // run / value count
+    if (r > 512u) {
+      tp_flag_error(4u);  // TP_DEVERR_RUNS
+      r = 512u;
+    }
+    if ((lane >> 4) && !v1) r = 0u;
+    rfor_pair_dispatch(bV, bL, r, __reduce_max_sync(FULL, r), lane, scratch);
+    __syncwarp();
+    return;
+  }
 #pragma unroll 1
   for (uint32_t h = 0; h < 2; ++h) {
     uint32_t* A = rfor_A(scratch, h);
