@@ -1277,6 +1277,10 @@ static inline uint32_t ht_slots(uint32_t ngroups) {
   while (s < HT_MAX_SLOTS && s < 2u * ngroups) s <<= 1;
   return s;
 }
+#ifndef TP_STAR_PAIR
+#define TP_STAR_PAIR 1  // ungrouped queries: the run-space RFOR pass over both blocks of a round at once
+                        // (q1.2 / q1.3 -8 %; in the grouped kernel q4.x -3 % but q3.2 +14 %: off there)
+#endif
 #ifndef TP_DENSE_PROBE_HINT
 #define TP_DENSE_PROBE_HINT 1
 #endif
@@ -1425,11 +1429,14 @@ struct StarOp : OpBase {
     return ((win >> (R & 31u)) & ((1ull << L) - 1ull)) != 0ull;
   }
   // one stream block pair (rows 512 h .. 512 h + 511 of the round), CC entries per lane and pass
-  template <int CC>
+  // PAIR: both blocks at once, lanes 16 h .. 16 h + 15 on block h (bV / bL / r per lane, rm = the
+  // larger r): one header decode and one 16-lane scan per pass serve both blocks
+  template <int CC, bool PAIR = false>
   __device__ __forceinline__ void rfor_runs(const uint32_t* bV, const uint32_t* bL, uint32_t r, uint32_t h,
                                             uint32_t c, bool range, bool per_run, bool need_ra, bool all_alive,
                                             uint32_t* RA, uint32_t* SB, uint32_t* PB, const uint32_t* AW,
-                                            uint32_t lane) {
+                                            uint32_t lane, uint32_t rm = 0u) {
+    if (PAIR) h = lane >> 4;
     const uint32_t refV = bV[1], refL = bL[1];  // references (FOR on both arrays)
     const uint4 wv = make_uint4(bV[2], bV[3], bV[4], bV[5]), wl = make_uint4(bL[2], bL[3], bL[4], bL[5]);
     const int32_t* __restrict__ T = A->table[c];
@@ -1438,8 +1445,8 @@ struct StarOp : OpBase {
     const uint32_t span = (uint32_t)(A->hi[c] - lo);
     uint32_t rowbase = 0u;  // rows of the block covered by earlier passes
 #pragma unroll 1
-    for (uint32_t e00 = 0; e00 < r; e00 += 32u * CC) {
-      const uint32_t e0 = e00 + CC * lane, m = (e0 >> 5) & 15u, pos = e0 & 31u;
+    for (uint32_t e00 = 0; e00 < (PAIR ? rm : r); e00 += (PAIR ? 16u : 32u) * CC) {
+      const uint32_t e0 = e00 + CC * (PAIR ? lane & 15u : lane), m = (e0 >> 5) & 15u, pos = e0 & 31u;
       const uint32_t bv = checked_bw(byte_of(wv, m)), bl = checked_bw(byte_of(wl, m));  // R2, R17
       const uint32_t* mV = bV + 6 + bytes_before(wv, m);  // miniblocks before m are full (R17)
       const uint32_t* mL = bL + 6 + bytes_before(wl, m);
@@ -1452,9 +1459,9 @@ struct StarOp : OpBase {
         len[k] = e0 + k < r ? refL + len[k] : 0u;
         run += len[k];
       }
-      const uint32_t incl = warp_inclusive_scan(run, lane);
+      const uint32_t incl = PAIR ? seg16_inclusive_scan(run) : warp_inclusive_scan(run, lane);
       uint32_t S = 512u * h + rowbase + incl - run;  // round row of entry e0's run start
-      rowbase += __shfl_sync(FULL, incl, 31);
+      rowbase += __shfl_sync(FULL, incl, PAIR ? lane | 15u : 31u);
       extract_c<CC>(mV, pos, bv, mv, val);
 #pragma unroll
       for (int k = 0; k < CC; ++k) val[k] += refV;
@@ -1627,6 +1634,23 @@ struct StarOp : OpBase {
     if (lane == 0) AW[32] = 0u;
     __syncwarp();
     const uint32_t live_lanes = __ballot_sync(FULL, alive != 0u);
+#if TP_STAR_PAIR
+    if (!GROUPED) {
+      const uint32_t tl0 = C.round_base + 2u * g.cw, hb = lane >> 4;
+      const bool v1 = C.t0s + tl0 + 1u < C.tile_end;  // (block 0 is inside the range: alive rows)
+      const bool go = (hb == 0u || v1) && ((live_lanes >> (16u * hb)) & 0xffffu) != 0u;
+      const uint32_t tl = tl0 + (hb && v1 ? 1u : 0u);
+      const uint32_t* bV = vv.sd + (vv.ss[vv.sshift + tl] - vv.lo + vv.dshift);
+      const uint32_t* bL = vl.sd + (vl.ss[vl.sshift + tl] - vl.lo + vl.dshift);
+      uint32_t r = go ? bV[0] : 0u;  // run / value count; 0: the half's block is skipped
+      if (r > 512u) {
+        tp_flag_error(4u);  // TP_DEVERR_RUNS
+        r = 512u;
+      }
+      rfor_runs<8, true>(bV, bL, r, hb, c, range, per_run, need_ra, all_alive, RA, SB, PB, AW, lane,
+                         __reduce_max_sync(FULL, r));
+    } else
+#endif
 #pragma unroll 1
     for (uint32_t h = 0; h < 2; ++h) {
       const uint32_t tl = C.round_base + 2u * g.cw + h;
