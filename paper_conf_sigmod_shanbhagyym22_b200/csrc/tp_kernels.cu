@@ -970,7 +970,7 @@ __device__ __forceinline__ void consumers_sync() {
 #define TP_SPARSE_LANE_MAX 8  // ... and (FOR filters / measures) the busiest lane's alive rows
 #endif
 #ifndef TP_RFOR_SPARSE_MAX
-#define TP_RFOR_SPARSE_MAX 32  // (<= 32: one alive row per lane)
+#define TP_RFOR_SPARSE_MAX 64  // (<= 64: up to two alive rows per lane; 64 vs 32: q3.1 -5 %, measured)
 #endif
 #ifndef TP_SPARSE_MAX
 #define TP_SPARSE_MAX 512  // alive rows (of a warp's 1024) at or below which a column goes sparse
@@ -1260,7 +1260,8 @@ struct StarArgs {
   uint32_t sparse_max;           // warp alive-row count at or below which a column is evaluated sparsely
   uint32_t sparse_lane_max;      // ... and the busiest lane's alive rows: the sparse loop runs for the
                                  // warp's maximum (alive rows cluster: runs of an order's lines)
-  uint32_t rfor_sparse_max;      // a GPU-RFOR column with at most this many alive rows (<= 32) in the
+  uint32_t hint_mask;            // bit c: column c's dense probes load with L1::no_allocate + L2 evict_last
+  uint32_t rfor_sparse_max;      // a GPU-RFOR column with at most this many alive rows (<= 64) in the
                                  // warp goes sparse (run lengths only + a binary search per row)
   long long* sums;
   unsigned long long* counts;
@@ -1283,6 +1284,10 @@ static inline uint32_t ht_slots(uint32_t ngroups) {
 #endif
 #ifndef TP_DENSE_PROBE_HINT
 #define TP_DENSE_PROBE_HINT 1
+#endif
+#ifndef TP_PROBE_HINT_MIN
+#define TP_PROBE_HINT_MIN 800000u  // table entries from which dense probes take the hint (SF20: the part table;
+                                  // the 600K-entry customer table loses with it, None q3.x +20-30 %, measured)
 #endif
 __device__ __forceinline__ int32_t probe_ld(const int32_t* p) { return __ldg(p); }
 // the dense probe of grouped queries (every alive row of a FOR / None column, the bulk of the
@@ -1533,7 +1538,7 @@ struct StarOp : OpBase {
     const Col& col = P.col[c];
     const StreamView vv = stream_view<true>(P, col.s0, C, 0), vl = stream_view<true>(P, col.s1, C, 1);
     uint32_t* RA = scratch + A->ra_off;  // run starts of both blocks (block h at 512 h)
-    uint32_t* LS = scratch + A->sb_off;  // the warp's alive rows, compacted (<= 32)
+    uint32_t* LS = scratch + A->sb_off;  // the warp's alive rows, compacted (<= 64)
     uint32_t* AW = LS + 66;              // alive words
     uint32_t* G = scratch + A->gs_off;
     uint32_t* W = scratch + A->ws_off;
@@ -1569,8 +1574,9 @@ struct StarOp : OpBase {
       rfor_starts(bL, r, lane, RA + 512u * h);
     }
     __syncwarp();
-    if (lane < nal) {
-      const uint32_t id = LS[lane], j = id >> 5, i = id & 31u, h = j >> 4;
+#pragma unroll 1
+    for (uint32_t t = lane; t < nal; t += 32u) {  // (up to 2 alive rows per lane)
+      const uint32_t id = LS[t], j = id >> 5, i = id & 31u, h = j >> 4;
       const uint32_t q = 32u * (j & 15u) + i;  // the row within its block
       const uint32_t* Sa = RA + 512u * h;
       uint32_t lo = 0u, hi = h ? r1 : r0;  // the last run starting at or before q (row 0 starts run 0)
@@ -1748,10 +1754,18 @@ struct StarOp : OpBase {
         const int32_t* __restrict__ T = A->table[c];
         const uint32_t kmin = (uint32_t)A->key_min[c], len = A->table_len[c];
         const uint32_t m = alive;
+        if (GROUPED && ((A->hint_mask >> c) & 1u)) {  // a table larger than L1 (host's choice)
 #pragma unroll
-        for (int i = 0; i < 32; ++i) {
-          const uint32_t kk = v[i] - kmin;
-          v[i] = ((m >> i) & 1u) && kk < len ? (uint32_t)(GROUPED ? dense_probe_ld(T + kk) : probe_ld(T + kk)) : 0xffffffffu;
+          for (int i = 0; i < 32; ++i) {
+            const uint32_t kk = v[i] - kmin;
+            v[i] = ((m >> i) & 1u) && kk < len ? (uint32_t)dense_probe_ld(T + kk) : 0xffffffffu;
+          }
+        } else {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) {
+            const uint32_t kk = v[i] - kmin;
+            v[i] = ((m >> i) & 1u) && kk < len ? (uint32_t)probe_ld(T + kk) : 0xffffffffu;
+          }
         }
         dense_payload(c, v, G, lane);
       } else {
@@ -2539,12 +2553,18 @@ tp_status tp_star_query(const tp_column* dcols, const tp_star_col* roles, int nc
     A.mstage[c] = roles[c].role == TP_ROLE_MEASURE && c != ncols - 1;
   }
   A.gzero = grouped && !gseen;
+  // dense probes into a table too large for L1 bypass it and stay in L2 (evict_last); smaller
+  // tables (supplier, date) keep their L1 hits
+  uint32_t hint_min = TP_PROBE_HINT_MIN;
+  if (const char* e = getenv("TILEPACK_PROBE_HINT_MIN")) hint_min = (uint32_t)atoi(e);  // tuning
+  for (int c = 0; c < ncols; ++c)
+    if (roles[c].role == TP_ROLE_PROBE && roles[c].table_len >= hint_min) A.hint_mask |= 1u << c;
   A.agg = agg;
   A.ngroups = ngroups;
   A.sparse_max = TP_SPARSE_MAX;
   A.sparse_lane_max = TP_SPARSE_LANE_MAX;
   A.rfor_sparse_max = TP_RFOR_SPARSE_MAX;
-  if (const char* e = getenv("TILEPACK_RFOR_SPARSE_MAX")) A.rfor_sparse_max = std::min(32, atoi(e));  // tests
+  if (const char* e = getenv("TILEPACK_RFOR_SPARSE_MAX")) A.rfor_sparse_max = std::min(64, atoi(e));  // tests
   if (const char* e = getenv("TILEPACK_SPARSE_LANE_MAX")) A.sparse_lane_max = (uint32_t)atoi(e);  // tuning
   if (const char* e = getenv("TILEPACK_SPARSE_MAX")) A.sparse_max = (uint32_t)atoi(e);  // tests: force a mode
   const uint32_t hts = grouped ? ht_slots(ngroups) : 0u;

@@ -18,7 +18,8 @@ def child(queries):
     from paper_conf_sigmod_shanbhagyym22_b200.ssb import QUERIES, SSBEngine
     g = json.load(open(os.path.join(ROOT, "tests", "golden", "ssb_sf20.json")))
     db = gen.generate(20, seed=5000, columns=gen.QUERY_COLUMNS)
-    eng = SSBEngine(db)
+    scheme = os.environ.get("TILEPACK_AB_SCHEME")  # "none": the uncompressed columns through the same kernel
+    eng = SSBEngine(db, schemes={c: scheme for c in gen.QUERY_COLUMNS} if scheme else None)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     res = {}
     for q in (queries or QUERIES):
@@ -52,15 +53,17 @@ if __name__ == "__main__":
         i = args.index("--queries")
         qs = args[i + 1]
         args = args[:i] + args[i + 2:]
-    for lib in args:
+    for spec in args:  # LIB or LIB:VAR=VAL,VAR=VAL (tuning knobs read from the environment)
+        lib, _, kv = spec.partition(":")
         env = dict(os.environ, TILEPACK_LIB_OVERRIDE=os.path.abspath(lib))
+        env.update(dict(x.split("=", 1) for x in kv.split(",") if x))
         out = subprocess.run([sys.executable, __file__, "--child", qs], env=env, capture_output=True, text=True)
         line = [x for x in out.stdout.splitlines() if x.startswith("RESULT")]
         if not line:
-            print(os.path.basename(lib), "FAILED", out.stderr[-800:], flush=True)
+            print(os.path.basename(spec), "FAILED", out.stderr[-800:], flush=True)
             continue
         r = json.loads(line[0][7:])
         import math
         geo = math.exp(sum(math.log(v[0]) for v in r.values()) / len(r))
-        print(os.path.basename(lib), "geomean %.4f" % geo, "parity", all(v[1] for v in r.values()),
+        print(os.path.basename(spec), "geomean %.4f" % geo, "parity", all(v[1] for v in r.values()),
               " ".join(f"{q}:{v[0]}" for q, v in r.items()), flush=True)

@@ -2,7 +2,7 @@
 # One box, one commit: every measurement under profiles/ (outputs in gpurun_out/r2/, copied by hand
 # to profiles/r02_*).   gpurun --timeout 5400 -- 'bash scripts/refresh_profiles.sh'
 set -x
-R=gpurun_out/r2
+R=gpurun_out/r2f
 mkdir -p $R
 nvidia-smi -q -d CLOCK > $R/clocks.txt 2>&1
 timeout 1500 python -m pytest tests -m gpu -q > $R/gpu_tests.log 2>&1; echo "tests rc=$?"

@@ -116,7 +116,7 @@ def test_oracle_star_query_brute_force():
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("mode", ["dense", "sparse", "auto"])
+@pytest.mark.parametrize("mode", ["dense", "sparse", "sparse64", "auto"])
 def test_gpu_star_query_modes(mode, monkeypatch):
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
@@ -125,7 +125,8 @@ def test_gpu_star_query_modes(mode, monkeypatch):
     if mode != "auto":
         monkeypatch.setenv("TILEPACK_SPARSE_MAX", "0" if mode == "dense" else "1024")
         monkeypatch.setenv("TILEPACK_SPARSE_LANE_MAX", "0" if mode == "dense" else "32")
-        monkeypatch.setenv("TILEPACK_RFOR_SPARSE_MAX", "0" if mode == "dense" else "32")
+        # sparse64: up to two alive rows per lane in the sparse GPU-RFOR path
+        monkeypatch.setenv("TILEPACK_RFOR_SPARSE_MAX", {"dense": "0", "sparse": "32", "sparse64": "64"}[mode])
     _run_cases(torch, tp, N, (1, 2), mode)
 
 
