@@ -354,6 +354,28 @@ __device__ __forceinline__ uint64_t sum_mb(const uint32_t* __restrict__ w, uint3
   } while (todo);
   return r;
 }
+// two miniblocks per lane (rounds r, r + 1): one dispatch when all 64 share a bitwidth, the two
+// unpack-and-sum bodies straight-line so that their loads and shifts interleave
+#define TP_SCASE2(B) \
+  case B:            \
+    r = sum_fixed<B>(w0) + sum_fixed<B>(w1); break;
+__device__ __forceinline__ uint64_t sum_mb2(const uint32_t* __restrict__ w0, uint32_t b0,
+                                            const uint32_t* __restrict__ w1, uint32_t b1) {
+  const uint32_t bmin = __reduce_min_sync(FULL, min(b0, b1)), bmax = __reduce_max_sync(FULL, max(b0, b1));
+  uint64_t r = 0;
+  if (bmin == bmax) {
+    switch (bmin) {
+      TP_SCASE2(0) TP_SCASE2(1) TP_SCASE2(2) TP_SCASE2(3) TP_SCASE2(4) TP_SCASE2(5) TP_SCASE2(6) TP_SCASE2(7)
+      TP_SCASE2(8) TP_SCASE2(9) TP_SCASE2(10) TP_SCASE2(11) TP_SCASE2(12) TP_SCASE2(13) TP_SCASE2(14) TP_SCASE2(15)
+      TP_SCASE2(16) TP_SCASE2(17) TP_SCASE2(18) TP_SCASE2(19) TP_SCASE2(20) TP_SCASE2(21) TP_SCASE2(22) TP_SCASE2(23)
+      TP_SCASE2(24) TP_SCASE2(25) TP_SCASE2(26) TP_SCASE2(27) TP_SCASE2(28) TP_SCASE2(29) TP_SCASE2(30) TP_SCASE2(31)
+      default: r = sum_fixed<32>(w0) + sum_fixed<32>(w1); break;
+    }
+    return r;
+  }
+  return sum_mb(w0, b0) + sum_mb(w1, b1);
+}
+#undef TP_SCASE2
 #undef TP_SCASE
 
 // sum of the bitwidth bytes below byte j of one bitwidth word (Opt. 3, P:900-918:

@@ -229,6 +229,9 @@ __device__ __forceinline__ uint32_t rfor_f_pos(uint32_t s) { return s ^ (((s >> 
 #ifndef TP_RFOR_BALLOT_CARRY
 #define TP_RFOR_BALLOT_CARRY 1  // carries by ballot + one shuffle (runs of 4: -2.5 %, SSB -0.3 %, measured)
 #endif
+#ifndef TP_SUM_PAIR
+#define TP_SUM_PAIR 1  // LEAN GPU-FOR decode->sum: two rounds per step
+#endif
 #ifndef TP_GLOBAL_SINGLE_DFOR
 #define TP_GLOBAL_SINGLE_DFOR 1
 #endif
@@ -687,6 +690,14 @@ __device__ __forceinline__ void run_pipeline(const Params& P, Op& op) {
         if (Op::kProducerSpin) mbar_wait(&full[slot], phase); else mbar_wait_backoff(&full[slot], phase);
         for (uint32_t r = 0; r < nr; ++r, ++rc) {
           C.round_base = r * TPR;
+          if constexpr (Op::kPairRounds) {
+            if (r + 1 < nr) {  // two rounds at once: two independent miniblock chains per lane
+              op.col2(P, C, g);
+              ++r;
+              ++rc;
+              continue;
+            }
+          }
           op.begin(P, C, g);
           op.col(P, C, g, scratch, 0, rc);
           op.end(P, C, g);
@@ -997,6 +1008,7 @@ __device__ __forceinline__ uint32_t valid_rows(const Params& P, const StageCtx& 
 
 struct OpBase {
   static constexpr bool kProducerSpin = false;
+  static constexpr bool kPairRounds = false;  // single-column: col2() takes rounds r and r + 1 together
   static constexpr uint32_t kMask = ~0u;  // scheme mix the kernel carries (M_*)
   __device__ void cta_init(const Params&, uint32_t*) {}
   __device__ void begin(const Params&, const StageCtx&, const Lane&) {}
@@ -1011,10 +1023,44 @@ template <uint32_t MASK, bool LEAN = false>
 struct SumOp : OpBase {
   static constexpr uint32_t kMask = MASK;
   static constexpr bool kProducerSpin = MASK == M_FOR || MASK == M_FORNM;
+  static constexpr bool kPairRounds = TP_SUM_PAIR && LEAN && MASK == M_FOR;
   unsigned long long* out;
   uint64_t acc;
   uint32_t sv_t0s = 0xffffffffu;  // the item whose stream view is cached (FOR)
   StreamView sv;
+  // LEAN GPU-FOR, rounds r and r + 1 of the item (C.round_base = round r): the lane's two
+  // miniblocks' views and unpacks are independent chains the scheduler interleaves
+  __device__ void col2(const Params& P, StageCtx& C, const Lane& g) {
+    const Col& c = P.col[0];
+    if (C.t0s != sv_t0s) {
+      sv = stream_view(P, c.s0, C);
+      sv_t0s = C.t0s;
+    }
+    uint32_t tl;
+    bool tv;
+    const MbView m0 = for_mb(P, c, C, g, sv, tl, tv);
+    C.round_base += TPR;
+    const MbView m1 = for_mb(P, c, C, g, sv, tl, tv);
+    const uint32_t tend = C.t0s + C.round_base + TPR;  // the end of the second round
+    C.round_base -= TPR;
+    const bool full = tend <= C.tile_end && (uint64_t)tend * TILE_ROWS <= P.n;  // (CTA-uniform)
+    if (full) {
+      acc += sum_mb2(m0.w, m0.b, m1.w, m1.b) + (uint64_t)((int64_t)(int32_t)m0.ref * 32) +
+             (uint64_t)((int64_t)(int32_t)m1.ref * 32);
+    } else {
+      for (int h = 0; h < 2; ++h) {
+        C.round_base += h * TPR;
+        const MbView m = h ? m1 : m0;
+        const uint32_t alive = valid_rows(P, C, g);
+        C.round_base -= h * TPR;
+        uint32_t e[32];
+        unpack_mb(m.w, m.b, e);
+#pragma unroll
+        for (int i = 0; i < 32; ++i)
+          if (alive & (1u << i)) acc += (uint64_t)(int64_t)(int32_t)(m.ref + e[i]);
+      }
+    }
+  }
   __device__ void col(const Params& P, const StageCtx& C, const Lane& g, uint32_t* scratch, uint32_t, uint32_t) {
     const Col& c = P.col[0];
     if (MASK == M_FOR || MASK == M_FORNM) {
