@@ -49,6 +49,7 @@ from them by `scripts/profiles_readme.py`.
 | `r02_ssb_sf20.json`, `r02_ssb_sf20_none.json`, `r02_ssb_sf160.json` | `scripts/bench_ssb.py` — 13 queries, GPU-* (checked against the oracle) / None / SF160 |
 | `r02_star_*.txt` | ncu source hot spots and details of the star kernel (q1.1, q2.1, q3.1, q4.1) |
 | `r02_star_waits.txt` | `scripts/prof_waits.py` — per-column cycle split of the star kernel (profiling build) |
+| `r02_ncu_rfor_runs4_global_*.txt`, `r02_ncu_dfor_sorted_global_details.txt` | `ncu --set full` of RFOR (runs of 4) and DFOR (sorted-uniform) decode→global: occupancy, issue, bank conflicts, source hot spots |
 | `r0?_encode.json`, `r0?_random_access.json`, `r0?_cascaded_ablation.json`, `r0?_nomb_ablation.json`, `r01_waterfall_sf20.json` | encoder, random access, cascading / miniblock ablations, SSB waterfall |
 
 ## Headline (config 2, b = 16, 500M rows, decode fused into an int64 sum)
