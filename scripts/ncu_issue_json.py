@@ -61,9 +61,11 @@ def main():
     for a, b in alias.items():
         if a in res:
             res[b] = res[a]
-    out = {"what": "ncu (--clock-control none) per decode configuration, 500M rows, one launch each: "
-                   "scripts/issue_profile.sh", "configs": res}
     path = os.path.join(ROOT, "profiles", "r02_issue.json")
+    prev = json.load(open(path)).get("configs", {}) if os.path.exists(path) else {}
+    prev.update(res)  # a run over some configurations refreshes those and keeps the others
+    out = {"what": "ncu (--clock-control none) per decode configuration, 500M rows, one launch each: "
+                   "scripts/issue_profile.sh", "configs": prev}
     json.dump(out, open(path, "w"), indent=1)
     for k, v in res.items():
         print(k, {kk: (round(vv, 3) if isinstance(vv, float) else vv) for kk, vv in v.items() if "stalls" not in kk})
