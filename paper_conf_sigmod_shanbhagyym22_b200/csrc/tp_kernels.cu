@@ -229,8 +229,9 @@ __device__ __forceinline__ uint32_t rfor_f_pos(uint32_t s) { return s ^ (((s >> 
 #ifndef TP_RFOR_BALLOT_CARRY
 #define TP_RFOR_BALLOT_CARRY 1  // carries by ballot + one shuffle (runs of 4: -2.5 %, SSB -0.3 %, measured)
 #endif
-#ifndef TP_SUM32_RFOR
-#define TP_SUM32_RFOR 1  // RFOR decode->sum: 32-bit partial sums when a chunk's values are < 2^27
+#ifndef TP_SUM32
+#define TP_SUM32 1  // DFOR / RFOR decode->sum: two 32-bit halves when a chunk's values are < 2^28
+                    // (DFOR D1 -8 %, RFOR runs of 4 -6 %, measured)
 #endif
 #ifndef TP_SUM_PAIR
 #define TP_SUM_PAIR 1  // LEAN GPU-FOR decode->sum: two rounds per step
@@ -1123,17 +1124,21 @@ struct SumOp : OpBase {
       }
       if (alive == 0xffffffffu) {  // per-lane branch, no collectives inside
         bool done = false;
-        if constexpr (TP_SUM32_RFOR && MASK == M_RFOR) {
-          // run values are usually small: when all 32 are below 2^27 (their OR says so) the 32-bit
-          // sum is exact -- one add per value instead of a 64-bit add and a sign count
-          uint32_t o = 0u, s32 = 0u;
+        if constexpr (TP_SUM32 && (MASK == M_RFOR || MASK == M_DFOR)) {
+          // decoded values below 2^28 (their OR says so: run values, keys of a 2^28 domain) sum
+          // exactly in two 32-bit halves of 16 -- one add per value instead of a 64-bit add and
+          // a sign count
+          uint32_t o = 0u;
 #pragma unroll
-          for (int i = 0; i < 32; ++i) {
-            o |= val[i];
-            s32 += val[i];
-          }
-          if ((o >> 27) == 0u) {
-            acc += s32;
+          for (int i = 0; i < 32; ++i) o |= val[i];
+          if ((o >> 28) == 0u) {
+            uint32_t sa = 0u, sb = 0u;
+#pragma unroll
+            for (int i = 0; i < 16; ++i) {
+              sa += val[i];
+              sb += val[16 + i];
+            }
+            acc += (uint64_t)sa + sb;
             done = true;
           }
         }
