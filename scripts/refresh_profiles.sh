@@ -1,6 +1,6 @@
 #!/bin/bash
-# One box, one commit: every measurement under profiles/ (outputs in gpurun_out/r2/, copied by hand
-# to profiles/r02_*).   gpurun --timeout 5400 -- 'bash scripts/refresh_profiles.sh'
+# One box, one commit: every measurement under profiles/ (outputs in gpurun_out/r2f/, copied by
+# scripts/collect_profiles.sh to profiles/r02_*).   gpurun --timeout 5400 -- 'bash scripts/refresh_profiles.sh'
 set -x
 R=gpurun_out/r2f
 mkdir -p $R
